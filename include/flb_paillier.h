@@ -1,0 +1,166 @@
+/* flb_paillier.h — C ABI of the B200 batched-Paillier library (FLBooster hot path).
+ *
+ * Paper: Zeng et al., "FLBooster: A Unified and Efficient Platform for Federated Learning
+ * Acceleration", ICDE 2023 — cited as PAPER L<line> of /root/reference/PAPER.md.
+ * This header is the boundary of SURVEY.md §8(b): Table I's Paillier rows (PAPER L252–L256:
+ * key_gen, encrypt, decrypt, add) batched over device pointers, plus scalar_mul, pack/unpack
+ * (PAPER §IV-B/§IV-C, Eq. 6–9) and a segmented ciphertext-product reduction.
+ *
+ * Conventions shared by every entry point
+ * ---------------------------------------
+ *  - Big integers are little-endian 32-bit limbs (base 2^w, w = 32), stored
+ *    row-major [count][words].  Plaintexts use pt_words = k/32 limbs and ciphertexts
+ *    ct_words = k/16 limbs, where k is the key's frame (1024, 2048, 3072 or 4096; smaller
+ *    "toy" keys are padded into the 1024 frame).  Buffers must be 16-byte aligned.
+ *  - Batch pointers are DEVICE pointers owned by the caller; every batch call is enqueued on
+ *    `stream` (a cudaStream_t passed as void*; NULL = legacy default stream) and returns
+ *    without synchronising.  The device is the caller's current CUDA device.  Scratch (window
+ *    tables, reduction partials) is taken from the device's stream-ordered pool on `stream`
+ *    and returned on the same stream.  Device faults surface at stream synchronisation.
+ *  - Key handles are immutable after creation and thread-safe; their constants are uploaded
+ *    to a device on first use there (a one-time synchronous copy).
+ *  - Status: FLB_OK (0) or a negative FLB_E* code; flb_last_error() gives a thread-local
+ *    message for the last failure.  Argument errors are detected before any launch.  Value
+ *    ranges (m < n, c < n^2, gcd(r, n) = 1) are NOT checked on the hot path: encrypt, add,
+ *    scalar_mul and reduce return the mathematical function of the given integers; decrypt is
+ *    specified for units c of Z_{n^2} (every unit is a valid ciphertext) and its
+ *    output for a non-unit is unspecified.
+ */
+#ifndef FLB_PAILLIER_H
+#define FLB_PAILLIER_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct flb_pub flb_pub;   /* n, n^2, Montgomery constants, encryption schedule */
+typedef struct flb_priv flb_priv; /* p, q, p^2, q^2, CRT constants, decryption schedules */
+
+enum {
+  FLB_OK = 0,
+  FLB_EINVAL = -1,      /* bad argument (null pointer, unsupported size, bad codec) */
+  FLB_ENOMEM = -2,      /* host or device allocation failed */
+  FLB_ECUDA = -3,       /* a CUDA call or kernel launch failed */
+  FLB_EKEY = -4,        /* key material rejected (not prime, p == q, gcd(n, phi) != 1) */
+  FLB_EUNSUPPORTED = -5 /* modulus larger than 4096 bits */
+};
+
+/* ---------------------------------------------------------------- keys (host, not timed) */
+
+/* Paillier::key_gen(size) (key generation L89).  Deterministic in `seed`:
+ * xoshiro256** candidates with the top two bits and the low bit set, small-prime sieve,
+ * 40-round Miller–Rabin.  key_bits in {1024, 2048, 3072, 4096}; p, q have
+ * key_bits/2 bits, bits(n) = key_bits, g = n + 1.  On success *pub and *priv are new handles
+ * (free with flb_pub_free / flb_priv_free).  Errors: FLB_EINVAL. */
+int flb_keygen(uint32_t key_bits, uint64_t seed, flb_pub** pub, flb_priv** priv);
+
+/* Import a key from its primes (host little-endian limbs, prime_words each).  The larger prime
+ * becomes p.  bits(n) <= 4096; keys below 1024 bits use the 1024 frame.  Errors: FLB_EINVAL
+ * (null / zero size), FLB_EKEY (p == q, a prime even or < 3, a prime failing Miller–Rabin,
+ * gcd(n, (p-1)(q-1)) != 1), FLB_EUNSUPPORTED (bits(n) > 4096). */
+int flb_key_from_primes(const uint32_t* p, const uint32_t* q, uint32_t prime_words,
+                        flb_pub** pub, flb_priv** priv);
+
+/* Copy p, q (prime_words(pub)= pt_words/2 limbs each) and n (pt_words limbs) to host
+ * buffers; any output pointer may be NULL. */
+int flb_key_export(const flb_priv* priv, uint32_t* p, uint32_t* q, uint32_t* n);
+
+void flb_pub_free(flb_pub* pub);
+void flb_priv_free(flb_priv* priv);
+
+uint32_t flb_key_bits(const flb_pub* pub);  /* bits(n) */
+uint32_t flb_pt_words(const flb_pub* pub);  /* frame/32 */
+uint32_t flb_ct_words(const flb_pub* pub);  /* frame/16 */
+/* floor((bits(n) - 1) / slot_bits): slots per plaintext that cannot wrap mod n (reading c16 of
+ * PAPER L258). */
+uint32_t flb_slot_capacity(const flb_pub* pub, uint32_t slot_bits);
+
+/* ---------------------------------------------------------------- batched device ops */
+
+/* Paillier::encrypt (Eq. 3): c_i = g^{m_i} r_i^n mod n^2 with g = n+1,
+ * computed as (1 + m_i n) r_i^n.  m: [count][pt_words], each m_i < n.  r: [count][pt_words]
+ * caller randomness (each r_i < n, gcd(r_i, n) = 1), or NULL to draw r_i on the device from
+ * Philox4x32-10 with key = seed and counter (ctr0 + i, j) exactly as oracle/philox.py draw_r
+ * (reading c4).  c: [count][ct_words].  count = 0 is a no-op.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_encrypt(const flb_pub* pub, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                uint64_t ctr0, uint32_t* c, size_t count, void* stream);
+
+/* Paillier::decrypt (Eq. 4), by CRT (reading c10).  c: [count][ct_words]
+ * (each a unit < n^2), m: [count][pt_words] receives m_i in [0, n).  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_decrypt(const flb_priv* priv, const uint32_t* c, uint32_t* m, size_t count, void* stream);
+
+/* Paillier::add (Eq. 5): out_i = c1_i * c2_i mod n^2.  All
+ * [count][ct_words]; out may alias c1 or c2.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_add(const flb_pub* pub, const uint32_t* c1, const uint32_t* c2, uint32_t* out,
+            size_t count, void* stream);
+
+/* Homomorphic scalar multiply (mod_pow; reading c19): out_i = c_i^{e_i} mod n^2
+ * = E(e_i m_i).  e: [count][e_words] unsigned little-endian exponents (1 <= e_words <= 128);
+ * e_i = 0 gives 1.  c, out: [count][ct_words] (no aliasing).  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_scalar_mul(const flb_pub* pub, const uint32_t* c, const uint32_t* e, uint32_t e_words,
+                   uint32_t* out, size_t count, void* stream);
+
+/* Segmented ciphertext product (Fig. 2 server aggregation; repeated Eq. 5):
+ * out_j = prod_{t = offsets[j]}^{offsets[j+1]-1} c[idx ? idx[t] : t] mod n^2, out_j = 1 for an
+ * empty segment.  c: [num_inputs][ct_words]; idx: device int64 [offsets[num_segments]] or
+ * NULL; offsets: device int64 [num_segments+1], non-decreasing, offsets[0] = 0.
+ * max_segment_len: an upper bound on any segment's length if known (sizes the number of
+ * reduction levels), 0 = unknown (num_inputs is used).  out: [num_segments][ct_words], must not
+ * alias c.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_reduce_segments(const flb_pub* pub, const uint32_t* c, size_t num_inputs,
+                        const int64_t* idx, const int64_t* offsets, size_t num_segments,
+                        size_t max_segment_len, uint32_t* out, void* stream);
+
+/* Encoding-quantisation + batch compression parameters (PAPER §IV-B/§IV-C):
+ * alpha: gradient bound (Eq. 6), qbits: r of Eq. 7 (L221, 1..52), pad_bits: b of Eq. 8
+ * (L223), slot_bits = qbits + pad_bits in {32, 64} (L331: "a multiple of 32"), slots: values
+ * per plaintext (1 <= slots <= flb_slot_capacity). */
+typedef struct {
+  double alpha;
+  uint32_t qbits, pad_bits, slot_bits, slots;
+} flb_codec;
+
+/* Quantise + pack (Eq. 6–9; readings c11, c13, c17): x: device float32 [n_values];
+ * pt: [ceil(n_values/slots)][pt_words]; plaintext j = sum_i q_{j*slots+i} 2^((slots-1-i) w).
+ * Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_pack(const flb_pub* pub, const flb_codec* codec, const float* x, size_t n_values,
+             uint32_t* pt, void* stream);
+
+/* Unpack + dequantise (reading c14): x_i = Sum_i / sigma - cnt * alpha in binary64,
+ * rounded to float32, with cnt = summands[i / slots] (device uint32 [num_pt]) or
+ * summands_scalar when summands is NULL.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_unpack(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt, size_t n_values,
+               const uint32_t* summands, uint32_t summands_scalar, float* x, void* stream);
+
+/* The exact slot integers Sum_i (device uint64 [n_values]).  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_unpack_sums(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt,
+                    size_t n_values, uint64_t* sums, void* stream);
+
+/* Debug entry for the Montgomery primitive (PAPER Alg. 2): out_i = a_i b_i R^-1
+ * mod n^2, R = 2^(32 ct_words), canonical.  a_i < n^2, b_i < n^2.  [count][ct_words]. */
+int flb_debug_mont_mul(const flb_pub* pub, const uint32_t* a, const uint32_t* b, uint32_t* out,
+                       size_t count, void* stream);
+
+/* Algorithmic cost of one element of an op, for roofline accounting: *mont_muls = Montgomery
+ * multiplications the kernel performs per element (window table, schedule, domain entry/exit),
+ * *limb_products = their CIOS limb-product count (2s^2 + s per s-limb multiplication, s^2 for
+ * the plain low-half product of the exact division).  op: 0 = encrypt (pub), 1 = decrypt
+ * (priv), 2 = add (pub), 3 = one reduce input (pub; excludes the per-chunk fix-up).
+ * Host only.  Errors: FLB_EINVAL. */
+int flb_op_cost(const flb_pub* pub, const flb_priv* priv, int op, uint64_t* mont_muls,
+                uint64_t* limb_products);
+
+/* Thread-local description of the last non-OK status ("" if none). */
+const char* flb_last_error(void);
+
+/* Library version string. */
+const char* flb_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* FLB_PAILLIER_H */

@@ -1,0 +1,274 @@
+"""flb-b200: batched Paillier homomorphic encryption for NVIDIA B200 (FLBooster hot path).
+
+Thin Python binding over the C ABI in ``include/flb_paillier.h`` (argument marshalling only —
+every step of the path runs in the CUDA kernels of ``csrc/``; there is no CPU fallback).
+PyTorch provides device memory and streams: batches are CUDA ``torch.int32`` tensors of shape
+``[count, words]`` holding little-endian 32-bit limbs, launched on
+``torch.cuda.current_stream()``.
+
+Paper: Zeng et al., "FLBooster", ICDE 2023 (``PAPER L<n>`` = /root/reference/PAPER.md line n).
+"""
+
+from __future__ import annotations
+
+import ctypes
+from typing import Optional, Tuple, Union
+
+import torch
+
+from . import _lib
+from ._lib import LIB, FlbError, check
+
+__all__ = [
+    "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "decrypt", "add",
+    "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
+    "Codec", "FlbError", "library_path", "op_cost",
+]
+
+library_path = _lib.LIB_PATH
+
+
+def _stream(stream: Optional[torch.cuda.Stream] = None) -> ctypes.c_void_p:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _ptr(t: Optional[torch.Tensor]) -> Optional[int]:
+    return None if t is None else t.data_ptr()
+
+
+def _check_batch(t: torch.Tensor, words: int, name: str) -> int:
+    if not t.is_cuda:
+        raise ValueError("%s must be a CUDA tensor" % name)
+    if t.dtype not in (torch.int32, torch.uint32):
+        raise ValueError("%s must be int32/uint32 limbs" % name)
+    if t.dim() != 2 or t.shape[1] != words or not t.is_contiguous():
+        raise ValueError("%s must be a contiguous [count, %d] tensor, got %s" % (name, words, tuple(t.shape)))
+    if t.data_ptr() % 16:
+        raise ValueError("%s must be 16-byte aligned" % name)
+    return t.shape[0]
+
+
+def _limbs_of(x: int, words: int):
+    arr = (ctypes.c_uint32 * words)()
+    for i in range(words):
+        arr[i] = (x >> (32 * i)) & 0xFFFFFFFF
+    return arr
+
+
+class PublicKey:
+    """Public key (n, g = n + 1): PAPER L89."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+        self.bits = LIB.flb_key_bits(handle)
+        self.pt_words = LIB.flb_pt_words(handle)
+        self.ct_words = LIB.flb_ct_words(handle)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def slot_capacity(self, slot_bits: int) -> int:
+        return LIB.flb_slot_capacity(self._h, slot_bits)
+
+    def __del__(self, _free=LIB.flb_pub_free):
+        h, self._h = getattr(self, "_h", None), None
+        if h:
+            _free(h)
+
+
+class PrivateKey:
+    """Private key (p, q): PAPER L89."""
+
+    def __init__(self, handle: ctypes.c_void_p, pub: PublicKey):
+        self._h = handle
+        self.pub = pub
+
+    @property
+    def handle(self):
+        return self._h
+
+    def export(self) -> Tuple[int, int, int]:
+        """(p, q, n) as Python ints, p > q."""
+        half = self.pub.pt_words // 2
+        p = (ctypes.c_uint32 * half)()
+        q = (ctypes.c_uint32 * half)()
+        n = (ctypes.c_uint32 * self.pub.pt_words)()
+        check("flb_key_export", LIB.flb_key_export(self._h, p, q, n))
+        to_int = lambda a: sum(int(w) << (32 * i) for i, w in enumerate(a))
+        return to_int(p), to_int(q), to_int(n)
+
+    def __del__(self, _free=LIB.flb_priv_free):
+        h, self._h = getattr(self, "_h", None), None
+        if h:
+            _free(h)
+
+
+def keygen(key_bits: int, seed: int) -> Tuple[PublicKey, PrivateKey]:
+    """Paillier::key_gen: deterministic host key generation."""
+    pub, priv = ctypes.c_void_p(), ctypes.c_void_p()
+    check("flb_keygen", LIB.flb_keygen(key_bits, seed & 0xFFFFFFFFFFFFFFFF, ctypes.byref(pub), ctypes.byref(priv)))
+    P = PublicKey(pub)
+    return P, PrivateKey(priv, P)
+
+
+def key_from_primes(p: int, q: int) -> Tuple[PublicKey, PrivateKey]:
+    """Import a key from its primes (e.g. the oracle's, for parity tests)."""
+    words = max((max(p, q).bit_length() + 31) // 32, 1)
+    pub, priv = ctypes.c_void_p(), ctypes.c_void_p()
+    check("flb_key_from_primes", LIB.flb_key_from_primes(_limbs_of(p, words), _limbs_of(q, words), words,
+                                                         ctypes.byref(pub), ctypes.byref(priv)))
+    P = PublicKey(pub)
+    return P, PrivateKey(priv, P)
+
+
+def encrypt(pub: PublicKey, m: torch.Tensor, r: Optional[torch.Tensor] = None, seed: int = 0, ctr0: int = 0,
+            out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """Paillier::encrypt (Eq. 3): c = (1 + m n) r^n mod n^2; r = Philox(seed, ctr0 + i) if None."""
+    M = _check_batch(m, pub.pt_words, "m")
+    if r is not None:
+        _check_batch(r, pub.pt_words, "r")
+    if out is None:
+        out = torch.empty((M, pub.ct_words), dtype=torch.int32, device=m.device)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_encrypt", LIB.flb_encrypt(pub.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0, _ptr(out), M,
+                                         _stream(stream)))
+    return out
+
+
+def decrypt(priv: PrivateKey, c: torch.Tensor, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """Paillier::decrypt (Eq. 4) by CRT."""
+    pub = priv.pub
+    M = _check_batch(c, pub.ct_words, "c")
+    if out is None:
+        out = torch.empty((M, pub.pt_words), dtype=torch.int32, device=c.device)
+    _check_batch(out, pub.pt_words, "out")
+    check("flb_decrypt", LIB.flb_decrypt(priv.handle, _ptr(c), _ptr(out), M, _stream(stream)))
+    return out
+
+
+def add(pub: PublicKey, c1: torch.Tensor, c2: torch.Tensor, out: Optional[torch.Tensor] = None,
+        stream=None) -> torch.Tensor:
+    """Paillier::add (Eq. 5): c1 c2 mod n^2."""
+    M = _check_batch(c1, pub.ct_words, "c1")
+    if _check_batch(c2, pub.ct_words, "c2") != M:
+        raise ValueError("c1 and c2 differ in count")
+    if out is None:
+        out = torch.empty_like(c1)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_add", LIB.flb_add(pub.handle, _ptr(c1), _ptr(c2), _ptr(out), M, _stream(stream)))
+    return out
+
+
+def scalar_mul(pub: PublicKey, c: torch.Tensor, e: torch.Tensor, out: Optional[torch.Tensor] = None,
+               stream=None) -> torch.Tensor:
+    """c^e mod n^2 = E(e m) (mod_pow); e: [count, e_words] unsigned limbs."""
+    M = _check_batch(c, pub.ct_words, "c")
+    if e.dim() != 2 or e.shape[0] != M:
+        raise ValueError("e must be [count, e_words]")
+    _check_batch(e, e.shape[1], "e")
+    if out is None:
+        out = torch.empty_like(c)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_scalar_mul", LIB.flb_scalar_mul(pub.handle, _ptr(c), _ptr(e), e.shape[1], _ptr(out), M,
+                                               _stream(stream)))
+    return out
+
+
+def reduce_segments(pub: PublicKey, c: torch.Tensor, offsets: torch.Tensor, idx: Optional[torch.Tensor] = None,
+                    max_segment_len: int = 0, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """out[j] = prod_{t in [off[j], off[j+1])} c[idx[t]] mod n^2 (empty = 1)."""
+    L = _check_batch(c, pub.ct_words, "c")
+    if offsets.dtype != torch.int64 or not offsets.is_cuda or offsets.dim() != 1 or not offsets.is_contiguous():
+        raise ValueError("offsets must be a contiguous CUDA int64 vector")
+    S = offsets.shape[0] - 1
+    if idx is not None and (idx.dtype != torch.int64 or not idx.is_cuda or not idx.is_contiguous()):
+        raise ValueError("idx must be a contiguous CUDA int64 vector")
+    if out is None:
+        out = torch.empty((S, pub.ct_words), dtype=torch.int32, device=c.device)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_reduce_segments", LIB.flb_reduce_segments(pub.handle, _ptr(c), L, _ptr(idx), _ptr(offsets), S,
+                                                         max_segment_len, _ptr(out), _stream(stream)))
+    return out
+
+
+class Codec:
+    """Encoding-quantisation / batch-compression parameters (PAPER §IV-B, §IV-C)."""
+
+    def __init__(self, alpha: float, qbits: int, pad_bits: int, slots: int):
+        self.alpha, self.qbits, self.pad_bits, self.slots = float(alpha), int(qbits), int(pad_bits), int(slots)
+        self.slot_bits = self.qbits + self.pad_bits
+
+    def struct(self) -> _lib.CodecStruct:
+        return _lib.CodecStruct(self.alpha, self.qbits, self.pad_bits, self.slot_bits, self.slots)
+
+    def num_plaintexts(self, n_values: int) -> int:
+        return -(-n_values // self.slots)
+
+
+def pack(pub: PublicKey, codec: Codec, x: torch.Tensor, out: Optional[torch.Tensor] = None,
+         stream=None) -> torch.Tensor:
+    """Quantise + pack float32 values into plaintexts (Eq. 6–9)."""
+    if not x.is_cuda or x.dtype != torch.float32 or x.dim() != 1 or not x.is_contiguous():
+        raise ValueError("x must be a contiguous CUDA float32 vector")
+    M = codec.num_plaintexts(x.shape[0])
+    if out is None:
+        out = torch.empty((M, pub.pt_words), dtype=torch.int32, device=x.device)
+    _check_batch(out, pub.pt_words, "out")
+    cs = codec.struct()
+    check("flb_pack", LIB.flb_pack(pub.handle, ctypes.byref(cs), _ptr(x), x.shape[0], _ptr(out), _stream(stream)))
+    return out
+
+
+def unpack(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int,
+           summands: Union[int, torch.Tensor] = 1, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """Unpack + dequantise: x = Sum/sigma - cnt*alpha (float64 -> float32)."""
+    _check_batch(pt, pub.pt_words, "pt")
+    if out is None:
+        out = torch.empty((n_values,), dtype=torch.float32, device=pt.device)
+    cs = codec.struct()
+    if isinstance(summands, torch.Tensor):
+        if summands.dtype not in (torch.int32, torch.uint32) or not summands.is_cuda:
+            raise ValueError("summands must be a CUDA int32 vector")
+        sp, ss = _ptr(summands), 0
+    else:
+        sp, ss = None, int(summands)
+    check("flb_unpack", LIB.flb_unpack(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, sp, ss, _ptr(out),
+                                       _stream(stream)))
+    return out
+
+
+def unpack_sums(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int, out: Optional[torch.Tensor] = None,
+                stream=None) -> torch.Tensor:
+    """The exact slot integers (int64 view of uint64)."""
+    _check_batch(pt, pub.pt_words, "pt")
+    if out is None:
+        out = torch.empty((n_values,), dtype=torch.int64, device=pt.device)
+    cs = codec.struct()
+    check("flb_unpack_sums", LIB.flb_unpack_sums(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, _ptr(out),
+                                                 _stream(stream)))
+    return out
+
+
+OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3}
+
+
+def op_cost(key, op: str) -> Tuple[int, int]:
+    """(Montgomery multiplications, CIOS limb products) per element of ``op`` (roofline accounting)."""
+    mm, lp = ctypes.c_uint64(), ctypes.c_uint64()
+    pub = key.handle if isinstance(key, PublicKey) else None
+    priv = key.handle if isinstance(key, PrivateKey) else None
+    check("flb_op_cost", LIB.flb_op_cost(pub, priv, OPS[op], ctypes.byref(mm), ctypes.byref(lp)))
+    return mm.value, lp.value
+
+
+def debug_mont_mul(pub: PublicKey, a: torch.Tensor, b: torch.Tensor, out: Optional[torch.Tensor] = None,
+                   stream=None) -> torch.Tensor:
+    """a b R^-1 mod n^2 (the Montgomery primitive of PAPER Alg. 2)."""
+    M = _check_batch(a, pub.ct_words, "a")
+    _check_batch(b, pub.ct_words, "b")
+    if out is None:
+        out = torch.empty_like(a)
+    check("flb_debug_mont_mul", LIB.flb_debug_mont_mul(pub.handle, _ptr(a), _ptr(b), _ptr(out), M, _stream(stream)))
+    return out

@@ -1,0 +1,729 @@
+// flb_api.cu — the C ABI (include/flb_paillier.h): key objects, constant derivation, launch
+// configuration and dispatch by key frame (layer L3).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/flb_paillier.h"
+#include "flb_kernels.cuh"
+#include "host_bn.hpp"
+
+using flb::host::Limbs;
+namespace H = flb::host;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+#define FLB_CK(call)                                                                    \
+  do {                                                                                  \
+    cudaError_t e_ = (call);                                                            \
+    if (e_ != cudaSuccess) return fail(FLB_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+constexpr int kBlock = 128;
+constexpr int kReduceChunk = 64;  // inputs per group in one reduction level
+
+// ----------------------------------------------------------------------------- constant blobs
+// All device constants of a key live in one buffer; Blob records word offsets.
+struct Blob {
+  std::vector<uint32_t> words;
+  size_t put(const Limbs& v, size_t w) {
+    // 16-byte align every array (uint4 loads)
+    while (words.size() % 4) words.push_back(0);
+    const size_t off = words.size();
+    Limbs r = H::resized(v, w);
+    words.insert(words.end(), r.begin(), r.end());
+    return off;
+  }
+  size_t put_raw(const std::vector<uint32_t>& v) {
+    while (words.size() % 4) words.push_back(0);
+    const size_t off = words.size();
+    words.insert(words.end(), v.begin(), v.end());
+    return off;
+  }
+};
+
+struct DevBlob {
+  std::mutex mu;
+  std::map<int, uint32_t*> per_dev;
+  ~DevBlob() {
+    for (auto& kv : per_dev) {
+      int cur;
+      if (cudaGetDevice(&cur) == cudaSuccess) {
+        cudaSetDevice(kv.first);
+        cudaFree(kv.second);
+        cudaSetDevice(cur);
+      }
+    }
+  }
+  // device copy of `b` on the current device (uploaded once)
+  int get(const Blob& b, uint32_t** out) {
+    int dev;
+    FLB_CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = per_dev.find(dev);
+    if (it != per_dev.end()) { *out = it->second; return FLB_OK; }
+    uint32_t* p = nullptr;
+    FLB_CK(cudaMalloc(&p, b.words.size() * 4));
+    FLB_CK(cudaMemcpy(p, b.words.data(), b.words.size() * 4, cudaMemcpyHostToDevice));
+    per_dev[dev] = p;
+    *out = p;
+    return FLB_OK;
+  }
+};
+
+int frame_for_bits(size_t nbits) {
+  if (nbits <= 1024) return 1024;
+  if (nbits <= 2048) return 2048;
+  if (nbits <= 3072) return 3072;
+  if (nbits <= 4096) return 4096;
+  return 0;
+}
+
+}  // namespace
+
+// ----------------------------------------------------------------------------- key structs
+struct flb_pub {
+  uint32_t nbits = 0, frame = 0, s = 0, sp = 0;
+  Limbs n, n2;
+  uint32_t n2_n0inv = 0;
+  H::Schedule enc;
+  Blob blob;
+  size_t o_n2 = 0, o_R2 = 0, o_R1 = 0, o_nR = 0, o_RL = 0, o_sched = 0;
+  DevBlob dev;
+};
+
+struct flb_priv {
+  flb_pub* pub = nullptr;  // owned copy of the public half (for n / frame)
+  Limbs p, q;
+  struct Prime {
+    Limbs P, P2;
+    uint32_t P_n0inv, P2_n0inv;
+    H::Schedule sched;
+    size_t o_P, o_P2, o_R2, o_R3, o_Pinv, o_hR, o_sched;
+  } pr[2];
+  size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
+  uint32_t n_n0inv = 0;
+  Blob blob;
+  DevBlob dev;
+  ~flb_priv() { delete pub; }
+};
+
+namespace {
+
+flb_pub* make_pub(const Limbs& n_in) {
+  auto* K = new flb_pub();
+  K->nbits = (uint32_t)H::bits(n_in);
+  K->frame = (uint32_t)frame_for_bits(K->nbits);
+  K->s = K->frame / 16;
+  K->sp = K->frame / 32;
+  K->n = H::resized(n_in, K->sp);
+  K->n2 = H::resized(H::mul(K->n, K->n), K->s);
+  H::MontCtx C(K->n2);
+  K->n2_n0inv = C.n0inv;
+  K->enc = H::best_schedule(K->n, 7);
+  K->o_n2 = K->blob.put(K->n2, K->s);
+  K->o_R2 = K->blob.put(C.R2, K->s);
+  K->o_R1 = K->blob.put(C.R1, K->s);
+  K->o_nR = K->blob.put(C.to(K->n), K->s);
+  // R^L mod n^2 for L = 0..kReduceChunk
+  std::vector<uint32_t> rl;
+  Limbs cur(K->s, 0);
+  cur[0] = 1;
+  cur = H::mod(cur, K->n2);
+  for (int L = 0; L <= kReduceChunk; L++) {
+    rl.insert(rl.end(), cur.begin(), cur.end());
+    cur = H::mont(cur, C.R2, K->n2, C.n0inv);  // * R
+  }
+  K->o_RL = K->blob.put_raw(rl);
+  K->o_sched = K->blob.put_raw(K->enc.ops);
+  return K;
+}
+
+flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
+  Limbs p = p_in, q = q_in;
+  if (H::cmp(p, q) < 0) std::swap(p, q);
+  const Limbs n = H::mul(p, q);
+  auto* V = new flb_priv();
+  V->pub = make_pub(n);
+  const uint32_t sp = V->pub->sp;
+  V->p = H::resized(p, sp);
+  V->q = H::resized(q, sp);
+  Limbs one(sp, 0);
+  one[0] = 1;
+  for (int i = 0; i < 2; i++) {
+    auto& R = V->pr[i];
+    const Limbs& P = i == 0 ? V->p : V->q;
+    const Limbs& Q = i == 0 ? V->q : V->p;
+    R.P = P;
+    R.P2 = H::resized(H::mul(P, P), sp);
+    H::MontCtx C2(R.P2), C1(R.P);
+    R.P2_n0inv = C2.n0inv;
+    R.P_n0inv = C1.n0inv;
+    Limbs pm1 = P;
+    H::sub_in(pm1, one);
+    R.sched = H::best_schedule(pm1, 7);
+    // h_P = (-Q)^-1 mod P
+    Limbs negQ = P;
+    H::sub_in(negQ, H::mod(Q, P));
+    const Limbs h = H::inv_mod_prime(negQ, P);
+    R.o_P2 = V->blob.put(R.P2, sp);
+    R.o_R2 = V->blob.put(C2.R2, sp);
+    R.o_R3 = V->blob.put(H::mont(C2.R2, C2.R2, R.P2, C2.n0inv) /* R^3 mod P^2 */, sp);
+    R.o_P = V->blob.put(P, sp);
+    R.o_Pinv = V->blob.put(H::inv_mod_2k(P, sp), sp);
+    R.o_hR = V->blob.put(C1.to(h), sp);
+    R.o_sched = V->blob.put_raw(R.sched.ops);
+  }
+  // CRT recombination constants
+  H::MontCtx Cn(V->pub->n), Cp(V->p);
+  V->n_n0inv = Cn.n0inv;
+  V->o_n = V->blob.put(V->pub->n, sp);
+  V->o_qR_n = V->blob.put(Cn.to(V->q), sp);
+  V->o_qinvR_p = V->blob.put(Cp.to(H::inv_mod_prime(V->q, V->p)), sp);
+  return V;
+}
+
+// ----------------------------------------------------------------------------- launching
+struct Pool {
+  static int prepare() {
+    static std::mutex mu;
+    static std::map<int, bool> done;
+    int dev;
+    FLB_CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    if (!done[dev]) {
+      cudaMemPool_t pool;
+      FLB_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+      uint64_t thr = ~0ull;
+      FLB_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+      done[dev] = true;
+    }
+    return FLB_OK;
+  }
+};
+
+template <typename K>
+int resident_blocks(K kernel, int* blocks) {
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, int> cache;
+  int dev;
+  FLB_CK(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair(dev, (const void*)kernel);
+  auto it = cache.find(key);
+  if (it != cache.end()) { *blocks = it->second; return FLB_OK; }
+  int per_sm = 0, sms = 0;
+  FLB_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kBlock, 0));
+  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  if (per_sm < 1) per_sm = 1;
+  cache[key] = per_sm * sms;
+  *blocks = per_sm * sms;
+  return FLB_OK;
+}
+
+// grid for `items` work units of T lanes each, capped at the resident capacity
+template <int T, typename K>
+int grid_for(K kernel, uint64_t items, int* grid) {
+  int cap;
+  int rc = resident_blocks(kernel, &cap);
+  if (rc) return rc;
+  const uint64_t want = (items * T + kBlock - 1) / kBlock;
+  *grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)cap));
+  return FLB_OK;
+}
+
+struct Scratch {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  ~Scratch() {
+    if (p) cudaFreeAsync(p, st);
+  }
+  int alloc(size_t bytes, cudaStream_t s) {
+    st = s;
+    if (bytes == 0) return FLB_OK;
+    int rc = Pool::prepare();
+    if (rc) return rc;
+    FLB_CK(cudaMallocAsync(&p, bytes, s));
+    return FLB_OK;
+  }
+};
+
+#define FLB_LAUNCH_CHECK() FLB_CK(cudaGetLastError())
+
+// ---- encrypt
+template <int X, int T>
+int run_encrypt(const flb_pub* K, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)K->enc.table * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::EncArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.nR = dev + K->o_nR;
+  A.sched = dev + K->o_sched;
+  A.sched_len = (int)K->enc.ops.size();
+  A.table = K->enc.table;
+  A.nbits = K->nbits;
+  A.pt_words = K->sp;
+  A.m = m;
+  A.r = r;
+  A.c = c;
+  A.count = count;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_decrypt(const flb_priv* V, const uint32_t* dev, const uint32_t* c, uint32_t* m, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_decrypt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->pr[0].sched.table, V->pr[1].sched.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->pub->sp * 4, st);
+  if (rc) return rc;
+  flb::DecArgs A;
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    A.pr[i].P2 = {dev + R.o_P2, R.P2_n0inv};
+    A.pr[i].R2 = dev + R.o_R2;
+    A.pr[i].R3 = dev + R.o_R3;
+    A.pr[i].P = {dev + R.o_P, R.P_n0inv};
+    A.pr[i].Pinv = dev + R.o_Pinv;
+    A.pr[i].hR = dev + R.o_hR;
+    A.pr[i].sched = dev + R.o_sched;
+    A.pr[i].sched_len = (int)R.sched.ops.size();
+    A.pr[i].table = R.sched.table;
+  }
+  A.n = {dev + V->o_n, V->n_n0inv};
+  A.qR_n = dev + V->o_qR_n;
+  A.qinvR_p = dev + V->o_qinvR_p;
+  A.c = c;
+  A.m = m;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_decrypt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T, bool DEBUG>
+int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
+            cudaStream_t st) {
+  auto kern = DEBUG ? flb::k_mont<X, T> : flb::k_add<X, T>;
+  int grid;
+  int rc = grid_for<T>(kern, count, &grid);
+  if (rc) return rc;
+  flb::AddArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.c1 = a;
+  A.c2 = b;
+  A.out = out;
+  A.count = count;
+  kern<<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_smul(const flb_pub* K, const uint32_t* dev, const uint32_t* c, const uint32_t* e, uint32_t e_words,
+             uint32_t* out, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_scalar_mul<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const uint32_t ebits = 32 * e_words;
+  const int bw = ebits <= 64 ? 3 : (ebits <= 512 ? 5 : 6);
+  Scratch sc;
+  rc = sc.alloc((size_t)(1u << bw) * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::SmulArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.R1 = dev + K->o_R1;
+  A.c = c;
+  A.e = e;
+  A.e_words = e_words;
+  A.bw = bw;
+  A.out = out;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_scalar_mul<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t num_inputs, const int64_t* idx,
+               const int64_t* offsets, size_t nseg, size_t max_len, uint32_t* out, cudaStream_t st) {
+  const int C = kReduceChunk;
+  if (max_len == 0) max_len = num_inputs;
+  int levels = 1;
+  for (size_t cap = C; cap < max_len; cap *= C) levels++;
+  // per-level buffers: chunk offsets [nseg+1], starts/ends [max_chunks], partials
+  const size_t max_chunks0 = num_inputs / C + nseg + 1;
+  Scratch s_plan, s_part0, s_part1;
+  const size_t plan_words = (nseg + 1) + 2 * max_chunks0;
+  int rc = s_plan.alloc(plan_words * sizeof(int64_t), st);
+  if (rc) return rc;
+  int64_t* chunk_off = (int64_t*)s_plan.p;
+  int64_t* cstart = chunk_off + (nseg + 1);
+  int64_t* cend = cstart + max_chunks0;
+  // partial buffers (ping-pong), sized for level 0 output
+  if (levels > 1) {
+    rc = s_part0.alloc(max_chunks0 * K->s * 4, st);
+    if (rc) return rc;
+    if (levels > 2) {
+      rc = s_part1.alloc((max_chunks0 / C + nseg + 1) * K->s * 4, st);
+      if (rc) return rc;
+    }
+  }
+  int grid_r;
+  rc = grid_for<T>(flb::k_reduce<X, T>, max_chunks0, &grid_r);
+  if (rc) return rc;
+  const uint32_t* in = c;
+  const int64_t* cur_idx = idx;
+  const int64_t* cur_off = offsets;
+  // level-(>0) offsets must survive while the next plan is built: keep two offset arrays
+  Scratch s_off;
+  rc = s_off.alloc(2 * (nseg + 1) * sizeof(int64_t), st);
+  if (rc) return rc;
+  int64_t* offbuf[2] = {(int64_t*)s_off.p, (int64_t*)s_off.p + (nseg + 1)};
+  size_t in_chunks = max_chunks0;
+  for (int lv = 0; lv < levels; lv++) {
+    flb::k_plan_scan<<<1, 1024, 0, st>>>(cur_off, (int64_t)nseg, C, chunk_off);
+    FLB_LAUNCH_CHECK();
+    const int fill_grid = (int)std::min<size_t>(4096, (in_chunks + 255) / 256 + 1);
+    flb::k_plan_fill<<<fill_grid, 256, 0, st>>>(cur_off, chunk_off, (int64_t)nseg, C, cstart, cend);
+    FLB_LAUNCH_CHECK();
+    const bool last = lv == levels - 1;
+    uint32_t* dst = last ? out : (uint32_t*)((lv % 2 == 0) ? s_part0.p : s_part1.p);
+    flb::RedArgs A;
+    A.N2 = {dev + K->o_n2, K->n2_n0inv};
+    A.R1 = dev + K->o_R1;
+    A.RL = dev + K->o_RL;
+    A.in = in;
+    A.idx = cur_idx;
+    A.cstart = cstart;
+    A.cend = cend;
+    A.nchunks = chunk_off + nseg;
+    A.out = dst;
+    A.max_chunks = in_chunks;
+    flb::k_reduce<X, T><<<grid_r, kBlock, 0, st>>>(A);
+    FLB_LAUNCH_CHECK();
+    if (!last) {
+      // next level: segments over this level's chunk partials
+      int64_t* nxt = offbuf[lv % 2];
+      FLB_CK(cudaMemcpyAsync(nxt, chunk_off, (nseg + 1) * sizeof(int64_t), cudaMemcpyDeviceToDevice, st));
+      cur_off = nxt;
+      in = dst;
+      cur_idx = nullptr;
+      in_chunks = in_chunks / C + nseg + 1;
+    }
+  }
+  return FLB_OK;
+}
+
+}  // namespace
+
+// ----------------------------------------------------------------------------- dispatch macros
+#define FLB_DISPATCH_ENC(frame, FN, ...)                              \
+  switch (frame) {                                                   \
+    case 1024: return FN<16, 4>(__VA_ARGS__);                        \
+    case 2048: return FN<16, 8>(__VA_ARGS__);                        \
+    case 3072: return FN<12, 16>(__VA_ARGS__);                       \
+    case 4096: return FN<16, 16>(__VA_ARGS__);                       \
+    default: return fail(FLB_EUNSUPPORTED, "unsupported key frame"); \
+  }
+#define FLB_DISPATCH_DEC(frame, FN, ...)                              \
+  switch (frame) {                                                   \
+    case 1024: return FN<16, 2>(__VA_ARGS__);                        \
+    case 2048: return FN<16, 4>(__VA_ARGS__);                        \
+    case 3072: return FN<12, 8>(__VA_ARGS__);                        \
+    case 4096: return FN<16, 8>(__VA_ARGS__);                        \
+    default: return fail(FLB_EUNSUPPORTED, "unsupported key frame"); \
+  }
+
+extern "C" {
+
+const char* flb_last_error(void) { return g_err.c_str(); }
+
+static uint64_t sched_mults(const H::Schedule& S) {
+  uint64_t m = (S.table > 1) ? (uint64_t)S.table : 0;  // x^2 + (table-1) products
+  for (size_t i = 1; i < S.ops.size(); i++) m += (S.ops[i] & 0xffffu) + ((S.ops[i] >> 16) ? 1 : 0);
+  return m;
+}
+
+int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls, uint64_t* limb_products) {
+  if (!mont_muls || !limb_products) return fail(FLB_EINVAL, "null output");
+  const flb_pub* P = K ? K : (V ? V->pub : nullptr);
+  if (!P) return fail(FLB_EINVAL, "null key");
+  const uint64_t s = P->s, sp = P->sp, cs = 2 * s * s + s, csp = 2 * sp * sp + sp;
+  switch (op) {
+    case 0: {  // encrypt: to-Montgomery, table + schedule, m n, final product
+      const uint64_t mm = 1 + sched_mults(P->enc) + 2;
+      *mont_muls = mm;
+      *limb_products = mm * cs;
+      return FLB_OK;
+    }
+    case 1: {  // decrypt: per prime 2 (entry) + table + schedule + 1 (exit) + 1 (h_P); mul_lo; CRT 2
+      if (!V) return fail(FLB_EINVAL, "decrypt cost needs the private key");
+      uint64_t mm = 2, lp = 0;
+      for (int i = 0; i < 2; i++) {
+        mm += 2 + sched_mults(V->pr[i].sched) + 1 + 1;
+        lp += sp * sp;  // exact division (low half product)
+      }
+      *mont_muls = mm;
+      *limb_products = mm * csp + lp;
+      return FLB_OK;
+    }
+    case 2:
+      *mont_muls = 2;
+      *limb_products = 2 * cs;
+      return FLB_OK;
+    case 3:
+      *mont_muls = 1;
+      *limb_products = cs;
+      return FLB_OK;
+  }
+  return fail(FLB_EINVAL, "unknown op");
+}
+const char* flb_version(void) { return "flb-b200 0.1 (sm_100a)"; }
+
+int flb_keygen(uint32_t key_bits, uint64_t seed, flb_pub** pub, flb_priv** priv) {
+  if (!pub || !priv) return fail(FLB_EINVAL, "null output pointer");
+  if (key_bits != 1024 && key_bits != 2048 && key_bits != 3072 && key_bits != 4096)
+    return fail(FLB_EINVAL, "key_bits must be 1024, 2048, 3072 or 4096");
+  try {
+    H::Xoshiro256 rng(seed);
+    for (;;) {
+      Limbs p = H::random_prime(key_bits / 2, rng), q = H::random_prime(key_bits / 2, rng);
+      if (H::cmp(p, q) == 0) continue;
+      Limbs n = H::mul(p, q);
+      if (H::bits(n) != key_bits) continue;
+      flb_priv* V = make_priv(p, q);
+      *priv = V;
+      *pub = make_pub(V->pub->n);
+      return FLB_OK;
+    }
+  } catch (const std::bad_alloc&) {
+    return fail(FLB_ENOMEM, "host allocation failed");
+  } catch (const std::exception& ex) {
+    return fail(FLB_EKEY, ex.what());
+  }
+}
+
+int flb_key_from_primes(const uint32_t* p, const uint32_t* q, uint32_t prime_words, flb_pub** pub, flb_priv** priv) {
+  if (!p || !q || !pub || !priv || prime_words == 0) return fail(FLB_EINVAL, "null pointer or zero size");
+  try {
+    Limbs P(p, p + prime_words), Q(q, q + prime_words);
+    if (H::cmp(P, Q) == 0) return fail(FLB_EKEY, "p == q");
+    if (!(P[0] & 1) || !(Q[0] & 1) || H::bits(P) < 2 || H::bits(Q) < 2) return fail(FLB_EKEY, "primes must be odd and >= 3");
+    const Limbs n = H::mul(P, Q);
+    if (H::bits(n) > 4096) return fail(FLB_EUNSUPPORTED, "bits(n) > 4096");
+    H::Xoshiro256 rng(0x5eed);
+    if (!H::probable_prime(P, rng, 20) || !H::probable_prime(Q, rng, 20)) return fail(FLB_EKEY, "a prime failed Miller-Rabin");
+    // gcd(n, (p-1)(q-1)) = 1  <=>  p does not divide q-1 and q does not divide p-1
+    Limbs one(prime_words, 0);
+    one[0] = 1;
+    Limbs pm1 = P, qm1 = Q;
+    H::sub_in(pm1, one);
+    H::sub_in(qm1, one);
+    if (H::is_zero(H::mod(qm1, P)) || H::is_zero(H::mod(pm1, Q))) return fail(FLB_EKEY, "gcd(n, phi(n)) != 1");
+    size_t pw = prime_words;
+    while (pw > 1 && P[pw - 1] == 0 && Q[pw - 1] == 0) pw--;
+    flb_priv* V = make_priv(H::resized(P, pw), H::resized(Q, pw));
+    *priv = V;
+    *pub = make_pub(V->pub->n);
+    return FLB_OK;
+  } catch (const std::bad_alloc&) {
+    return fail(FLB_ENOMEM, "host allocation failed");
+  } catch (const std::exception& ex) {
+    return fail(FLB_EKEY, ex.what());
+  }
+}
+
+int flb_key_export(const flb_priv* V, uint32_t* p, uint32_t* q, uint32_t* n) {
+  if (!V) return fail(FLB_EINVAL, "null key");
+  const uint32_t half = V->pub->sp / 2;
+  if (p) for (uint32_t i = 0; i < half; i++) p[i] = V->p[i];
+  if (q) for (uint32_t i = 0; i < half; i++) q[i] = V->q[i];
+  if (n) for (uint32_t i = 0; i < V->pub->sp; i++) n[i] = V->pub->n[i];
+  return FLB_OK;
+}
+
+void flb_pub_free(flb_pub* pub) { delete pub; }
+void flb_priv_free(flb_priv* priv) { delete priv; }
+uint32_t flb_key_bits(const flb_pub* K) { return K ? K->nbits : 0; }
+uint32_t flb_pt_words(const flb_pub* K) { return K ? K->sp : 0; }
+uint32_t flb_ct_words(const flb_pub* K) { return K ? K->s : 0; }
+uint32_t flb_slot_capacity(const flb_pub* K, uint32_t slot_bits) {
+  return (K && slot_bits) ? (K->nbits - 1) / slot_bits : 0;
+}
+
+int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* c,
+                size_t count, void* stream) {
+  if (!K || !m || !c) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_ENC(K->frame, run_encrypt, K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+}
+
+int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count, void* stream) {
+  if (!V || !c || !m) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_DEC(V->pub->frame, run_decrypt, V, dev, c, m, count, (cudaStream_t)stream);
+}
+
+int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* out, size_t count, void* stream) {
+  if (!K || !c1 || !c2 || !out) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+#define RUN_ADD(X, T) run_add<X, T, false>(K, dev, c1, c2, out, count, (cudaStream_t)stream)
+  switch (K->frame) {
+    case 1024: return RUN_ADD(16, 4);
+    case 2048: return RUN_ADD(16, 8);
+    case 3072: return RUN_ADD(12, 16);
+    case 4096: return RUN_ADD(16, 16);
+  }
+#undef RUN_ADD
+  return fail(FLB_EUNSUPPORTED, "unsupported key frame");
+}
+
+int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
+                       void* stream) {
+  if (!K || !a || !b || !out) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+#define RUN_MONT(X, T) run_add<X, T, true>(K, dev, a, b, out, count, (cudaStream_t)stream)
+  switch (K->frame) {
+    case 1024: return RUN_MONT(16, 4);
+    case 2048: return RUN_MONT(16, 8);
+    case 3072: return RUN_MONT(12, 16);
+    case 4096: return RUN_MONT(16, 16);
+  }
+#undef RUN_MONT
+  return fail(FLB_EUNSUPPORTED, "unsupported key frame");
+}
+
+int flb_scalar_mul(const flb_pub* K, const uint32_t* c, const uint32_t* e, uint32_t e_words, uint32_t* out,
+                   size_t count, void* stream) {
+  if (!K || !c || !e || !out) return fail(FLB_EINVAL, "null pointer");
+  if (e_words < 1 || e_words > 128) return fail(FLB_EINVAL, "e_words must be in [1, 128]");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_ENC(K->frame, run_smul, K, dev, c, e, e_words, out, count, (cudaStream_t)stream);
+}
+
+int flb_reduce_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs, const int64_t* idx,
+                        const int64_t* offsets, size_t num_segments, size_t max_segment_len, uint32_t* out,
+                        void* stream) {
+  if (!K || !offsets || !out) return fail(FLB_EINVAL, "null pointer");
+  if (num_inputs > 0 && !c) return fail(FLB_EINVAL, "null input");
+  if (num_segments == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_ENC(K->frame, run_reduce, K, dev, c, num_inputs, idx, offsets, num_segments, max_segment_len, out,
+                   (cudaStream_t)stream);
+}
+
+static int codec_args(const flb_pub* K, const flb_codec* cd, flb::CodecArgs* A) {
+  if (!cd) return fail(FLB_EINVAL, "null codec");
+  if (cd->qbits < 1 || cd->qbits > 52) return fail(FLB_EINVAL, "qbits must be in [1, 52]");
+  if (cd->slot_bits != cd->qbits + cd->pad_bits) return fail(FLB_EINVAL, "slot_bits != qbits + pad_bits");
+  if (cd->slot_bits != 32 && cd->slot_bits != 64) return fail(FLB_EINVAL, "slot_bits must be 32 or 64");
+  if (cd->slots < 1 || cd->slots > flb_slot_capacity(K, cd->slot_bits))
+    return fail(FLB_EINVAL, "slots must be in [1, floor((bits(n)-1)/slot_bits)]");
+  if (!(cd->alpha > 0.0)) return fail(FLB_EINVAL, "alpha must be > 0");
+  A->alpha = cd->alpha;
+  A->sigma = (double)((1ull << cd->qbits) - 1) / (2.0 * cd->alpha);
+  A->qbits = cd->qbits;
+  A->slot_words = cd->slot_bits / 32;
+  A->slots = cd->slots;
+  A->pt_words = K->sp;
+  A->qmax = (1ull << cd->qbits) - 1;
+  return FLB_OK;
+}
+
+static int grid_1d(uint64_t n) {
+  int dev, sms = 148;
+  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint64_t want = (n + 255) / 256;
+  return (int)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)sms * 8));
+}
+
+int flb_pack(const flb_pub* K, const flb_codec* cd, const float* x, size_t n_values, uint32_t* pt, void* stream) {
+  if (!K || !x || !pt) return fail(FLB_EINVAL, "null pointer");
+  flb::CodecArgs A;
+  int rc = codec_args(K, cd, &A);
+  if (rc) return rc;
+  if (n_values == 0) return FLB_OK;
+  const uint64_t n_pt = (n_values + A.slots - 1) / A.slots;
+  flb::k_pack<<<grid_1d(n_pt * A.pt_words), 256, 0, (cudaStream_t)stream>>>(x, n_values, n_pt, A, pt);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+int flb_unpack(const flb_pub* K, const flb_codec* cd, const uint32_t* pt, size_t n_values, const uint32_t* summands,
+               uint32_t summands_scalar, float* x, void* stream) {
+  if (!K || !x || !pt) return fail(FLB_EINVAL, "null pointer");
+  flb::CodecArgs A;
+  int rc = codec_args(K, cd, &A);
+  if (rc) return rc;
+  if (n_values == 0) return FLB_OK;
+  flb::k_unpack<<<grid_1d(n_values), 256, 0, (cudaStream_t)stream>>>(pt, n_values, A, summands, summands_scalar, x);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+int flb_unpack_sums(const flb_pub* K, const flb_codec* cd, const uint32_t* pt, size_t n_values, uint64_t* sums,
+                    void* stream) {
+  if (!K || !sums || !pt) return fail(FLB_EINVAL, "null pointer");
+  flb::CodecArgs A;
+  int rc = codec_args(K, cd, &A);
+  if (rc) return rc;
+  if (n_values == 0) return FLB_OK;
+  flb::k_unpack_sums<<<grid_1d(n_values), 256, 0, (cudaStream_t)stream>>>(pt, n_values, A,
+                                                                          (unsigned long long*)sums);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+}  // extern "C"

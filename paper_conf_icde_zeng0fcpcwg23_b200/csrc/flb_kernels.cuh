@@ -1,0 +1,562 @@
+// flb_kernels.cuh — the batched Paillier / codec kernels (layers L1, L2) for sm_100a.
+//
+// Every kernel is a persistent grid: a fixed number of thread groups (sized from occupancy, see
+// flb_api.cu) loops over the batch.  A warp's groups always take the same number of trips, so
+// the shuffles/ballots of flb_bn.cuh never see an inactive lane; elements past the end compute
+// on zeros and skip their store.  Exponent schedules shared by the batch (n for encryption,
+// p-1 and q-1 for decryption) are read warp-uniformly, so control flow never diverges.
+#pragma once
+#include <cstdint>
+#include "flb_bn.cuh"
+
+namespace flb {
+
+struct ModRef {
+  const uint32_t* n;  // modulus limbs in the kernel's frame
+  uint32_t n0inv;     // -n^-1 mod 2^32 (reading c6)
+};
+
+// ----------------------------------------------------------------------------- group indexing
+template <int T>
+struct Grid {
+  uint32_t gid, G, wg0;
+  int k;
+  __device__ __forceinline__ Grid() {
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    gid = tid / T;
+    G = (gridDim.x * blockDim.x) / T;
+    wg0 = (tid & ~31u) / T;
+    k = (int)(threadIdx.x & (T - 1));
+  }
+};
+
+template <int X, int T>
+__device__ __forceinline__ void load_mod(uint32_t (&n)[X], const ModRef& M) {
+  const int k = (int)(lane_id() & (T - 1));
+  load_limbs<X>(n, M.n + k * X);
+}
+
+template <int X, int T>
+__device__ __forceinline__ void load_const(uint32_t (&r)[X], const uint32_t* p) {
+  const int k = (int)(lane_id() & (T - 1));
+  load_limbs<X>(r, p + k * X);
+}
+
+template <int X, int T>
+__device__ __forceinline__ void set_one(uint32_t (&r)[X]) {
+  const int k = (int)(lane_id() & (T - 1));
+  zero_limbs<X>(r);
+  if (k == 0) r[0] = 1;
+}
+
+// Load limbs [k*X, k*X+X) of an element with `words` limbs (words may be < X*T: the rest are 0).
+template <int X, int T>
+__device__ __forceinline__ void load_elem(uint32_t (&r)[X], const uint32_t* base, uint32_t words, bool valid) {
+  const int k = (int)(lane_id() & (T - 1));
+  if (valid && (uint32_t)(k * X) < words) load_limbs<X>(r, base + k * X);
+  else zero_limbs<X>(r);
+}
+
+// ----------------------------------------------------------------------------- Philox4x32-10
+// Reading c4: r_i = Philox4x32-10(key = seed, ctr = (i lo, i hi, j, 0)), word 4j+t of r.
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 key) {
+#pragma unroll
+  for (int r = 0; r < 10; r++) {
+    if (r) { key.x += 0x9E3779B9u; key.y += 0xBB67AE85u; }
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ key.x, lo1, hi0 ^ c.w ^ key.y, lo0);
+  }
+  return c;
+}
+
+// r for element `index`: pt_words Philox words, bits >= nbits-1 cleared, 0 -> 1.
+template <int X, int T>
+__device__ __forceinline__ void philox_r(uint32_t (&r)[X], uint64_t seed, uint64_t index, uint32_t pt_words,
+                                         uint32_t nbits) {
+  const int k = (int)(lane_id() & (T - 1));
+  const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
+#pragma unroll
+  for (int v = 0; v < X / 4; v++) {
+    const uint32_t w0 = (uint32_t)(k * X + 4 * v);
+    uint4 o = make_uint4(0, 0, 0, 0);
+    if (w0 < pt_words) o = philox4x32_10(make_uint4((uint32_t)index, (uint32_t)(index >> 32), w0 / 4, 0), key);
+    r[4 * v] = o.x; r[4 * v + 1] = o.y; r[4 * v + 2] = o.z; r[4 * v + 3] = o.w;
+  }
+  const uint32_t lim = nbits - 1;  // keep bits [0, nbits-1)
+#pragma unroll
+  for (int j = 0; j < X; j++) {
+    const uint32_t w = (uint32_t)(k * X + j);
+    if (w >= pt_words || 32u * w >= lim) r[j] = 0;
+    else if (32u * (w + 1) > lim) r[j] &= (1u << (lim - 32u * w)) - 1u;
+  }
+  const bool nz = !all_zero<X>(r);
+  const uint32_t bal = __ballot_sync(FULL, nz);
+  const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
+  const uint32_t gm = (T == 32) ? 0xffffffffu : (((1u << T) - 1u) << base);
+  if ((bal & gm) == 0 && k == 0) r[0] = 1;
+}
+
+// ----------------------------------------------------------------------------- modexp
+// Sliding-window Montgomery exponentiation with a batch-shared schedule (host_bn.hpp
+// sliding_schedule).  x: base in Montgomery form (clobbered).  The odd-power table lives in
+// global scratch: entry i of this group at tab + i*stride + k*X.
+template <int X, int T>
+__device__ __forceinline__ void modexp_sched(uint32_t (&acc)[X], uint32_t (&x)[X], const uint32_t* __restrict__ sched,
+                                             int len, int table, uint32_t* tab, size_t stride,
+                                             const uint32_t (&n)[X], uint32_t n0inv) {
+  const int k = (int)(lane_id() & (T - 1));
+  uint32_t b[X];
+  store_limbs<X>(tab + k * X, x);
+  if (table > 1) {
+    mont_mul<X, T>(b, x, x, n, n0inv);
+#pragma unroll 1
+    for (int i = 1; i < table; i++) {
+      mont_mul<X, T>(x, x, b, n, n0inv);
+      store_limbs<X>(tab + (size_t)i * stride + k * X, x);
+    }
+  }
+  const uint32_t op0 = __ldg(sched);
+  load_limbs_plain<X>(acc, tab + (size_t)((op0 >> 16) - 1) * stride + k * X);
+#pragma unroll 1
+  for (int o = 1; o < len; o++) {
+    const uint32_t op = __ldg(sched + o);
+    const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
+    const int steps = sq + (idx >= 0 ? 1 : 0);
+#pragma unroll 1
+    for (int i = 0; i < steps; i++) {
+      if (i == sq) {
+        load_limbs_plain<X>(b, tab + (size_t)idx * stride + k * X);
+      } else {
+#pragma unroll
+        for (int j = 0; j < X; j++) b[j] = acc[j];
+      }
+      mont_mul<X, T>(acc, acc, b, n, n0inv);
+    }
+  }
+}
+
+// ----------------------------------------------------------------------------- encrypt
+struct EncArgs {
+  ModRef N2;               // n^2 in the s-limb frame
+  const uint32_t* R2;      // R^2 mod n^2
+  const uint32_t* nR;      // n*R mod n^2
+  const uint32_t* sched;   // schedule of the exponent n
+  int sched_len, table;
+  uint32_t nbits, pt_words;
+  const uint32_t* m;       // [count][pt_words]
+  const uint32_t* r;       // [count][pt_words] or null (Philox)
+  uint32_t* c;             // [count][2*pt_words]
+  uint64_t count, seed, ctr0;
+  uint32_t* scratch;       // table * G * S words
+};
+
+// c = (1 + m n) r^n mod n^2 (Eq. 3 with g = n+1: g^m = 1 + m n mod n^2).
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_encrypt(const EncArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  const uint32_t n0inv = A.N2.n0inv;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t x[X], b[X], acc[X];
+    if (A.r) load_elem<X, T>(x, A.r + e * A.pt_words, A.pt_words, valid);
+    else philox_r<X, T>(x, A.seed, A.ctr0 + e, A.pt_words, A.nbits);
+    load_const<X, T>(b, A.R2);
+    mont_mul<X, T>(x, x, b, n, n0inv);                       // r~ = r R mod n^2
+    modexp_sched<X, T>(acc, x, A.sched, A.sched_len, A.table, tab, stride, n, n0inv);  // r^n R
+    load_elem<X, T>(x, A.m + e * A.pt_words, A.pt_words, valid);
+    load_const<X, T>(b, A.nR);
+    mont_mul<X, T>(x, x, b, n, n0inv);                       // m n (< n^2, exact)
+    grp_add_small<X, T>(x, 1u);                              // 1 + m n
+    mont_mul<X, T>(acc, acc, x, n, n0inv);                   // r^n (1 + m n)
+    if (valid) store_limbs<X>(A.c + e * S + g.k * X, acc);
+  }
+}
+
+// ----------------------------------------------------------------------------- decrypt (CRT)
+struct PrimeArgs {
+  ModRef P2;              // P^2 in the sp frame
+  const uint32_t* R2;     // R^2 mod P^2
+  const uint32_t* R3;     // R^3 mod P^2
+  ModRef P;               // P in the sp frame
+  const uint32_t* Pinv;   // P^-1 mod 2^(32 sp)
+  const uint32_t* hR;     // h_P R mod P, h_p = (-q)^-1 mod p, h_q = (-p)^-1 mod q
+  const uint32_t* sched;  // schedule of P-1
+  int sched_len, table;
+};
+struct DecArgs {
+  PrimeArgs pr[2];        // [0] = p (the larger prime), [1] = q
+  ModRef n;               // n in the sp frame
+  const uint32_t* qR_n;   // q R mod n
+  const uint32_t* qinvR_p;// q^-1 R mod p
+  const uint32_t* c;      // [count][2 sp]
+  uint32_t* m;            // [count][sp]
+  uint64_t count;
+  uint32_t* scratch;      // max table * G * sp
+};
+
+// m = D(c) (Eq. 4) by CRT (reading c10):
+//   m_P = L_P(c^(P-1) mod P^2) h_P mod P, m = m_q + q ((m_p - m_q) q^-1 mod p).
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_decrypt(const DecArgs A) {
+  constexpr int S = X * T;  // sp
+  const Grid<T> g;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t mres[2][X];
+#pragma unroll 1
+    for (int P = 0; P < 2; P++) {
+      const PrimeArgs& pa = A.pr[P];
+      uint32_t n[X], lo[X], hi[X], b[X], x[X];
+      load_mod<X, T>(n, pa.P2);
+      load_elem<X, T>(lo, A.c + e * (2 * S), S, valid);
+      load_elem<X, T>(hi, A.c + e * (2 * S) + S, S, valid);
+      load_const<X, T>(b, pa.R2);
+      mont_mul<X, T>(lo, lo, b, n, pa.P2.n0inv);          // c_lo R mod P^2
+      load_const<X, T>(b, pa.R3);
+      mont_mul<X, T>(hi, hi, b, n, pa.P2.n0inv);          // c_hi R^2 mod P^2
+      const uint32_t cy = grp_add<X, T>(x, lo, hi);
+      grp_cond_sub<X, T>(x, n, cy);                       // c R mod P^2 (Montgomery form of c)
+      modexp_sched<X, T>(lo, x, pa.sched, pa.sched_len, pa.table, tab, stride, n, pa.P2.n0inv);
+      set_one<X, T>(b);
+      mont_mul<X, T>(lo, lo, b, n, pa.P2.n0inv);          // c^(P-1) mod P^2
+      grp_sub_one<X, T>(lo);                              // x - 1 = L * P
+      load_const<X, T>(b, pa.Pinv);
+      mul_lo<X, T>(hi, lo, b);                            // L = (x - 1) / P (exact division)
+      load_mod<X, T>(n, pa.P);
+      load_const<X, T>(b, pa.hR);
+      mont_mul<X, T>(mres[P], hi, b, n, pa.P.n0inv);      // m_P = L h_P mod P
+    }
+    uint32_t n[X], d[X], t[X];
+    load_mod<X, T>(n, A.pr[0].P);
+    const uint32_t br = grp_sub<X, T>(d, mres[0], mres[1]);   // m_p - m_q (m_q < q < p)
+#pragma unroll
+    for (int j = 0; j < X; j++) t[j] = br ? n[j] : 0u;
+    grp_add<X, T>(d, d, t);                                    // mod p
+    load_const<X, T>(t, A.qinvR_p);
+    mont_mul<X, T>(d, d, t, n, A.pr[0].P.n0inv);               // u = (m_p - m_q) q^-1 mod p
+    load_mod<X, T>(n, A.n);
+    load_const<X, T>(t, A.qR_n);
+    mont_mul<X, T>(d, d, t, n, A.n.n0inv);                     // q u (< n, exact)
+    grp_add<X, T>(d, d, mres[1]);                              // m = m_q + q u
+    if (valid) store_limbs<X>(A.m + e * S + g.k * X, d);
+  }
+}
+
+// ----------------------------------------------------------------------------- hom-add
+struct AddArgs {
+  ModRef N2;
+  const uint32_t* R2;
+  const uint32_t* c1;
+  const uint32_t* c2;
+  uint32_t* out;
+  uint64_t count;
+};
+
+// c1 c2 mod n^2 (Eq. 5) = mont(mont(c1, c2), R^2).
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_add(const AddArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t a[X], b[X];
+    load_elem<X, T>(a, A.c1 + e * S, S, valid);
+    load_elem<X, T>(b, A.c2 + e * S, S, valid);
+#pragma unroll 1
+    for (int it = 0; it < 2; it++) {
+      mont_mul<X, T>(a, a, b, n, A.N2.n0inv);
+      load_const<X, T>(b, A.R2);
+    }
+    if (valid) store_limbs<X>(A.out + e * S + g.k * X, a);
+  }
+}
+
+// ----------------------------------------------------------------------------- debug mont_mul
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_mont(const AddArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t a[X], b[X];
+    load_elem<X, T>(a, A.c1 + e * S, S, valid);
+    load_elem<X, T>(b, A.c2 + e * S, S, valid);
+    mont_mul<X, T>(a, a, b, n, A.N2.n0inv);
+    if (valid) store_limbs<X>(A.out + e * S + g.k * X, a);
+  }
+}
+
+// ----------------------------------------------------------------------------- scalar-mul
+struct SmulArgs {
+  ModRef N2;
+  const uint32_t* R2;      // R^2 mod n^2
+  const uint32_t* R1;      // R mod n^2 (Montgomery one)
+  const uint32_t* c;       // [count][S]
+  const uint32_t* e;       // [count][e_words]
+  uint32_t e_words;
+  int bw;                  // fixed window width
+  uint32_t* out;
+  uint64_t count;
+  uint32_t* scratch;       // 2^bw * G * S
+};
+
+__device__ __forceinline__ uint32_t exp_window(const uint32_t* e, uint32_t e_words, int w, int bw) {
+  const uint32_t lo = (uint32_t)(w * bw), word = lo >> 5, off = lo & 31u;
+  uint32_t v = (word < e_words) ? __ldg(e + word) >> off : 0u;
+  if (off + bw > 32 && word + 1 < e_words) v |= __ldg(e + word + 1) << (32 - off);
+  return v & ((1u << bw) - 1u);
+}
+
+// c^e mod n^2 (mod_pow; reading c19), per-element exponent, fixed window with
+// an always-multiply step (table[0] = Montgomery one) so control flow is uniform.
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_scalar_mul(const SmulArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  const uint32_t n0inv = A.N2.n0inv;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  const int table = 1 << A.bw;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t el = base + (g.gid - g.wg0);
+    const bool valid = el < A.count;
+    uint32_t x[X], b[X], acc[X];
+    load_elem<X, T>(x, A.c + el * S, S, valid);
+    load_const<X, T>(b, A.R2);
+    mont_mul<X, T>(x, x, b, n, n0inv);
+    load_const<X, T>(acc, A.R1);
+    store_limbs<X>(tab + g.k * X, acc);
+    store_limbs<X>(tab + stride + g.k * X, x);
+#pragma unroll
+    for (int j = 0; j < X; j++) b[j] = x[j];
+#pragma unroll 1
+    for (int i = 2; i < table; i++) {
+      mont_mul<X, T>(b, b, x, n, n0inv);
+      store_limbs<X>(tab + (size_t)i * stride + g.k * X, b);
+    }
+    // highest window holding a set bit, maximised over the warp (uniform trip count)
+    const uint32_t* ep = A.e + el * A.e_words;
+    int top = -1;
+    if (valid) {
+      for (int w = (int)A.e_words - 1; w >= 0; w--) {
+        const uint32_t v = __ldg(ep + w);
+        if (v) { top = (int)((32 * w + 31 - __clz(v)) / A.bw); break; }
+      }
+    }
+    top = __reduce_max_sync(FULL, top);
+#pragma unroll 1
+    for (int w = top; w >= 0; w--) {
+      if (w != top) {
+#pragma unroll 1
+        for (int s = 0; s < A.bw; s++) {
+#pragma unroll
+          for (int j = 0; j < X; j++) b[j] = acc[j];
+          mont_mul<X, T>(acc, acc, b, n, n0inv);
+        }
+      }
+      const uint32_t d = valid ? exp_window(ep, A.e_words, w, A.bw) : 0u;
+      load_limbs_plain<X>(b, tab + (size_t)d * stride + g.k * X);
+      mont_mul<X, T>(acc, acc, b, n, n0inv);
+    }
+    set_one<X, T>(b);
+    mont_mul<X, T>(acc, acc, b, n, n0inv);
+    if (valid) store_limbs<X>(A.out + el * S + g.k * X, acc);
+  }
+}
+
+// ----------------------------------------------------------------------------- segmented reduce
+struct RedArgs {
+  ModRef N2;
+  const uint32_t* R1;          // R mod n^2
+  const uint32_t* RL;          // R^L mod n^2 for L = 0..C, [C+1][S]
+  const uint32_t* in;          // [*][S]
+  const int64_t* idx;          // gather index into `in` or null
+  const int64_t* cstart;       // per chunk: first input position
+  const int64_t* cend;         // per chunk: one past the last
+  const int64_t* nchunks;      // device scalar: number of chunks
+  uint32_t* out;               // [nchunks][S]
+  uint64_t max_chunks;         // host bound for the grid
+};
+
+// out[ch] = prod_{t in chunk} in[idx[t]] mod n^2.  acc starts at R (Montgomery one); after L
+// raw-input Montgomery products it is prod * R^-(L-1); one product with R^L mod n^2 removes the
+// factor.  Lanes whose chunk is shorter multiply by R mod n^2 (a no-op).
+template <int X, int T>
+__global__ void __launch_bounds__(128) k_reduce(const RedArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  const uint64_t count = (uint64_t)*A.nchunks;
+  for (uint64_t base = g.wg0; base < count; base += g.G) {
+    const uint64_t ch = base + (g.gid - g.wg0);
+    const bool valid = ch < count;
+    int64_t st = 0, len = 0;
+    if (valid) { st = A.cstart[ch]; len = A.cend[ch] - st; }
+    const int maxlen = __reduce_max_sync(FULL, (int)len);
+    uint32_t acc[X], b[X];
+    load_const<X, T>(acc, A.R1);
+#pragma unroll 1
+    for (int t = 0; t <= maxlen; t++) {
+      if (t < maxlen) {
+        if (t < len) {
+          const int64_t pos = A.idx ? A.idx[st + t] : st + t;
+          load_limbs<X>(b, A.in + (size_t)pos * S + g.k * X);
+        } else {
+          load_const<X, T>(b, A.R1);
+        }
+      } else {
+        load_const<X, T>(b, A.RL + (size_t)len * S);
+      }
+      mont_mul<X, T>(acc, acc, b, n, A.N2.n0inv);
+    }
+    if (valid) store_limbs<X>(A.out + ch * S + g.k * X, acc);
+  }
+}
+
+// chunk planning: chunks_j = max(1, ceil(len_j / C)); chunk_off = exclusive scan (one block).
+__global__ void k_plan_scan(const int64_t* __restrict__ offsets, int64_t nseg, int C, int64_t* __restrict__ chunk_off) {
+  __shared__ int64_t warp_sums[32];
+  __shared__ int64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (int64_t base = 0; base < nseg; base += blockDim.x) {
+    const int64_t j = base + threadIdx.x;
+    int64_t v = 0;
+    if (j < nseg) {
+      const int64_t len = offsets[j + 1] - offsets[j];
+      v = len <= 0 ? 1 : (len + C - 1) / C;
+    }
+    // inclusive warp scan
+    int64_t x = v;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) warp_sums[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      int64_t s = (lane < (int)(blockDim.x >> 5)) ? warp_sums[lane] : 0;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t y = __shfl_up_sync(FULL, s, o);
+        if (lane >= o) s += y;
+      }
+      warp_sums[lane] = s;  // inclusive over warps
+    }
+    __syncthreads();
+    const int64_t before = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
+    if (j < nseg) chunk_off[j] = before;
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) carry = before + v;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) chunk_off[nseg] = carry;
+}
+
+__global__ void k_plan_fill(const int64_t* __restrict__ offsets, const int64_t* __restrict__ chunk_off, int64_t nseg,
+                            int C, int64_t* __restrict__ cstart, int64_t* __restrict__ cend) {
+  const int64_t total = chunk_off[nseg];
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < total; c += (int64_t)gridDim.x * blockDim.x) {
+    // segment j: last j with chunk_off[j] <= c
+    int64_t lo = 0, hi = nseg - 1;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi + 1) >> 1;
+      if (chunk_off[mid] <= c) lo = mid; else hi = mid - 1;
+    }
+    const int64_t j = lo, r = c - chunk_off[j];
+    const int64_t s = offsets[j] + r * C;
+    int64_t e = s + C;
+    if (e > offsets[j + 1]) e = offsets[j + 1];
+    if (e < s) e = s;
+    cstart[c] = s;
+    cend[c] = e;
+  }
+}
+
+// ----------------------------------------------------------------------------- codec
+struct CodecArgs {
+  double alpha, sigma;
+  uint32_t qbits, slot_words, slots, pt_words;
+  uint64_t qmax;
+};
+
+// Eq. 6–7 in binary64, op for op as oracle/codec.py quantize (reading c11, c13).
+__device__ __forceinline__ uint64_t quantize(float xf, const CodecArgs& C) {
+  double x = (double)xf;
+  if (isnan(x)) x = 0.0;
+  x = fmin(fmax(x, -C.alpha), C.alpha);
+  const double e = __dadd_rn(x, C.alpha);
+  const double p = __dmul_rn(e, C.sigma);
+  double q = rint(p);
+  if (q < 0.0) q = 0.0;
+  uint64_t qi = (uint64_t)q;
+  return qi > C.qmax ? C.qmax : qi;
+}
+
+// pt[j] = sum_i q_{jS+i} 2^((S-1-i) w) (Eq. 9, reading c17); one thread per word.
+__global__ void k_pack(const float* __restrict__ x, uint64_t n_values, uint64_t n_pt, CodecArgs C,
+                       uint32_t* __restrict__ pt) {
+  const uint64_t total = n_pt * C.pt_words;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t j = i / C.pt_words;
+    const uint32_t t = (uint32_t)(i - j * C.pt_words);
+    uint32_t w = 0;
+    if (t < C.slots * C.slot_words) {
+      const uint32_t slot = C.slots - 1 - t / C.slot_words, part = t % C.slot_words;
+      const uint64_t v = j * C.slots + slot;
+      if (v < n_values && part < 2) w = (uint32_t)(quantize(x[v], C) >> (32 * part));
+    }
+    pt[i] = w;
+  }
+}
+
+__device__ __forceinline__ uint64_t slot_value(const uint32_t* __restrict__ pt, uint64_t v, const CodecArgs& C) {
+  const uint64_t j = v / C.slots;
+  const uint32_t i = (uint32_t)(v - j * C.slots);
+  const uint32_t w0 = (C.slots - 1 - i) * C.slot_words;
+  const uint32_t* p = pt + j * C.pt_words + w0;
+  uint64_t s = p[0];
+  if (C.slot_words > 1) s |= (uint64_t)p[1] << 32;
+  return s;
+}
+
+// x = Sum / sigma - cnt alpha in binary64, then binary32 (reading c14).
+__global__ void k_unpack(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
+                         const uint32_t* __restrict__ summands, uint32_t summands_scalar, float* __restrict__ out) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n_values; v += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t s = slot_value(pt, v, C);
+    const uint32_t cnt = summands ? summands[v / C.slots] : summands_scalar;
+    const double t1 = __ddiv_rn(__ull2double_rn(s), C.sigma);
+    const double t2 = __dmul_rn((double)cnt, C.alpha);
+    out[v] = __double2float_rn(__dsub_rn(t1, t2));
+  }
+}
+
+__global__ void k_unpack_sums(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
+                              unsigned long long* __restrict__ out) {
+  for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n_values; v += (uint64_t)gridDim.x * blockDim.x)
+    out[v] = slot_value(pt, v, C);
+}
+
+}  // namespace flb
