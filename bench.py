@@ -1,0 +1,439 @@
+#!/usr/bin/env python
+"""bench.py — FLBooster hot path on B200: Paillier ops/s at 2048-bit keys (BASELINE.json metric).
+
+Workload (BASELINE.json configs[1], "C2"): Homo-LR gradient aggregation.  Per rank, 8 clients
+each hold a 1,048,576-element float32 gradient (synthetic, N(0, 0.05^2) clipped, 1 % at +-1).
+One step is one pass of the whole hot path:
+    pack (Eq. 6–9, w = 32, S = 63)  ->  encrypt 8 x 16,645 plaintexts (Eq. 3, Philox r)
+    ->  segmented product over clients (Eq. 5)  [N > 1: all_to_all + N-way product]
+    ->  CRT decrypt (Eq. 4)  ->  unpack + dequantise (L297, cnt = clients)
+metric value = (encryptions + decryptions + homomorphic additions) per second over all ranks.
+
+  python bench.py [--gpus N --steps K --warmup W]          # this library (CUDA)
+  python bench.py --impl reference                         # the CPU oracle on the host cores
+Multi-GPU: python -m torch.distributed.run --nproc-per-node N bench.py --gpus N ... (weak
+scaling: every rank hosts 8 clients of an 8N-client federation; rows are reduce-scattered).
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CLIENTS = 8            # clients per rank (C2: "summed over 8 clients")
+N_VALUES = 1 << 20     # gradient length (Avazu-sized)
+KEY_BITS = 2048
+KEY_SEED = 0xF1B0 + 2048
+ALPHA = 1.0
+SLOT_BITS = 32         # slots a multiple of 32 bits
+METRIC = "Paillier encrypt/decrypt/hom-add ops/sec at 2048-bit key, 1/2/4/8 B200"
+UNIT = "ops/s"
+PEAK_LP_PER_CLK_SM = 32  # IMAD.WIDE.U32(.X): half-rate FMA-heavy pipe (tools/imad_peak.cu)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["flb", "reference"], default="flb")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-sample-seconds", type=float, default=20.0)
+    return ap.parse_args()
+
+
+def codec_params(world: int):
+    participants = CLIENTS * world
+    pad = max(1, math.ceil(math.log2(participants)))  # b = ceil(log2 p)
+    return ALPHA, SLOT_BITS - pad, pad
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), "--query-gpu=" + self.FIELDS, "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx.append(float(parts[2]))
+                power.append(float(parts[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        loaded = [s for s in sm if s > 500] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "power_w_max": max(power) if power else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+# ----------------------------------------------------------------------------- CPU oracle timing
+def _oracle_enc(args):
+    from oracle import paillier, philox
+    n, m, seed, idx, ptw = args
+    return paillier.encrypt(n, m, philox.draw_r(n, seed, idx, ptw))
+
+
+def _oracle_dec(args):
+    from oracle import paillier
+    p, q, c = args
+    return paillier.decrypt(p, q, c)
+
+
+def oracle_rates(sample_seconds: float, cores: int):
+    """Time the oracle as it stands on the host cores (multiprocessing over a bounded sample).
+    Returns per-op wall seconds (with `cores` workers) and a description of the sample."""
+    import multiprocessing as mp
+    import random
+    import numpy as np
+    import synthetic
+    from oracle import codec, paillier
+    p, q = paillier.keygen(KEY_BITS, KEY_SEED)  # the oracle's own key of the same size
+    n = p * q
+    n2 = n * n
+    ptw = KEY_BITS // 32
+    rng = random.Random(1)
+    # size the sample from a single-op calibration so the whole leg takes ~sample_seconds
+    t0 = time.perf_counter()
+    _oracle_enc((n, rng.randrange(n), 7, 0, ptw))
+    t_enc1 = time.perf_counter() - t0
+    budget = sample_seconds * cores
+    n_enc = max(cores, int(0.7 * budget / t_enc1) // cores * cores)
+    n_dec = max(cores, n_enc // 2)
+    ms = [rng.randrange(n) for _ in range(n_enc)]
+    ctx = mp.get_context("fork")
+    with ctx.Pool(cores) as pool:
+        t0 = time.perf_counter()
+        cs = pool.map(_oracle_enc, [(n, ms[i], 7, i, ptw) for i in range(n_enc)], chunksize=1)
+        t_enc = (time.perf_counter() - t0) / n_enc
+        t0 = time.perf_counter()
+        pool.map(_oracle_dec, [(p, q, cs[i % n_enc]) for i in range(n_dec)], chunksize=1)
+        t_dec = (time.perf_counter() - t0) / n_dec
+    # hom-add (single process; microseconds each)
+    k = 2000
+    t0 = time.perf_counter()
+    acc = cs[0]
+    for i in range(k):
+        acc = paillier.add(n, acc, cs[i % n_enc])
+    t_add = (time.perf_counter() - t0) / k / cores  # embarrassingly parallel across cores
+    # codec: pack + unpack of a sample of one client's gradient
+    x = synthetic.c2_gradient(0)[: 63 * 64]
+    alpha, qb, pb = codec_params(1)
+    t0 = time.perf_counter()
+    z = codec.pack([float(v) for v in x], alpha, qb, pb, 63)
+    codec.unpack(z, len(x), alpha, qb, pb, 63, CLIENTS)
+    t_codec_value = (time.perf_counter() - t0) / len(x) / cores
+    sample = ("oracle (pure-Python ints): %d encryptions + %d CRT-free decryptions on %d processes, "
+              "%d hom-adds, pack+unpack of %d values; extrapolated to the C2 step mix"
+              % (n_enc, n_dec, cores, k, len(x)))
+    return {"t_enc": t_enc, "t_dec": t_dec, "t_add": t_add, "t_codec_value": t_codec_value, "sample": sample}
+
+
+def c2_step_ops(rows: int, world: int):
+    enc = CLIENTS * rows * world
+    adds = (CLIENTS - 1) * rows * world + (world - 1) * rows
+    dec = rows
+    return enc, dec, adds
+
+
+def oracle_value(r, rows: int):
+    enc, dec, adds = c2_step_ops(rows, 1)
+    step = enc * r["t_enc"] + dec * r["t_dec"] + adds * r["t_add"] + (CLIENTS + 1) * N_VALUES * r["t_codec_value"]
+    return (enc + dec + adds) / step, step
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    from oracle import codec
+    cores = cpu_cores()
+    rows = codec.num_plaintexts(N_VALUES, 63)
+    per = max(3.0, 60.0 / max(1, args.steps + args.warmup))
+    vals = []
+    for s in range(args.warmup + args.steps):
+        r = oracle_rates(per, cores)
+        v, step_s = oracle_value(r, rows)
+        if s >= args.warmup:
+            vals.append((v, step_s, r["sample"]))
+    v = statistics.median([x[0] for x in vals])
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.median([x[1] for x in vals]),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32-limb bigint (+f64 codec)",
+        "data": "synthetic",
+        "config": {"workload": "C2 Homo-LR aggregation, 2048-bit key, 8 clients x 1,048,576 values",
+                   "note": "CPU oracle: each step times a bounded sample and extrapolates to the C2 step"},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": vals[-1][2]},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------- CUDA arm
+def run_flb(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+
+    import paper_conf_icde_zeng0fcpcwg23_b200 as flb
+    from paper_conf_icde_zeng0fcpcwg23_b200 import dist as fdist
+    import synthetic
+
+    pub, priv = flb.keygen(KEY_BITS, KEY_SEED)  # product keygen (C++ host), same key on every rank
+    alpha, qbits, pad = codec_params(world)
+    S = pub.slot_capacity(SLOT_BITS)            # 63 at 2048 bits (reading c16)
+    cd = flb.Codec(alpha, qbits, pad, S)
+    rows = cd.num_plaintexts(N_VALUES)          # 16,645
+    rows_p = fdist.padded_rows(rows, world)
+    rpr = rows_p // world
+    ptw, ctw = pub.pt_words, pub.ct_words
+
+    # inputs resident in HBM before timing
+    grads_host = [torch.from_numpy(synthetic.c2_gradient(CLIENTS * rank + c)) for c in range(CLIENTS)]
+    grads = [g.to(dev) for g in grads_host]
+    offs, idx = fdist.client_segments(CLIENTS, rows, rows_p, device=dev)
+    pt = torch.empty((CLIENTS * rows, ptw), dtype=torch.int32, device=dev)
+    ct = torch.empty((CLIENTS * rows, ctw), dtype=torch.int32, device=dev)
+    part = torch.empty((rows_p, ctw), dtype=torch.int32, device=dev)
+    recv = torch.empty_like(part)
+    fin = torch.empty((rpr, ctw), dtype=torch.int32, device=dev)
+    dec = torch.empty((rpr, ptw), dtype=torch.int32, device=dev)
+    r0, r1 = fdist.rank_rows(rows, world, rank)
+    my_values = max(0, min(N_VALUES, r1 * S) - r0 * S)
+    out = torch.empty((max(my_values, 1),), dtype=torch.float32, device=dev)
+    foffs, fidx = fdist.finish_segments(world, rpr, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def reduce_cb(buf, o, i, L):
+        return flb.reduce_segments(pub, buf, o, idx=i, max_segment_len=L, out=fin)
+
+    ev = {}
+
+    def mark(name):
+        e = torch.cuda.Event(enable_timing=True)
+        e.record()
+        ev.setdefault(name, []).append(e)
+
+    def step(s, gsrc=None):
+        seed = 0xC2000000 + s
+        mark("t0")
+        for c in range(CLIENTS):
+            flb.pack(pub, cd, grads[c] if gsrc is None else gsrc[c], out=pt[c * rows:(c + 1) * rows])
+        mark("t_pack")
+        flb.encrypt(pub, pt, seed=seed, ctr0=rank * CLIENTS * rows, out=ct)
+        mark("t_enc")
+        flb.reduce_segments(pub, ct, offs, idx=idx, max_segment_len=CLIENTS, out=part)
+        mark("t_red")
+        if world > 1:
+            fdist.exchange_and_finish(part, None, reduce_cb, world, recv=recv)
+            agg = fin
+        else:
+            agg = part
+        mark("t_xchg")
+        flb.decrypt(priv, agg[: (r1 - r0) if world > 1 else rows], out=dec[: (r1 - r0) if world > 1 else rows])
+        mark("t_dec")
+        if my_values:
+            flb.unpack(pub, cd, dec, my_values, summands=CLIENTS * world, out=out[:my_values])
+        mark("t_unpack")
+
+    ops_enc, ops_dec, ops_add = c2_step_ops(rows, world)
+    total_ops = ops_enc + ops_dec + ops_add
+
+    for s in range(args.warmup):
+        step(s)
+    torch.cuda.synchronize()
+    ev.clear()
+
+    clocks = ClockSampler(torch.cuda.current_device() if world == 1 else local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    step_ms = []
+    for s in range(args.steps):
+        flush.zero_()
+        step(1000 + s)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+
+    names = ["t0", "t_pack", "t_enc", "t_red", "t_xchg", "t_dec", "t_unpack"]
+    phase = {n: 0.0 for n in names[1:]}
+    for s in range(args.steps):
+        step_ms.append(ev["t0"][s].elapsed_time(ev["t_unpack"][s]))
+        for a, b in zip(names[:-1], names[1:]):
+            phase[b] += ev[a][s].elapsed_time(ev[b][s]) / args.steps
+    ms = sum(step_ms) / len(step_ms)
+    if world > 1:
+        t = torch.tensor([ms] + [phase[n] for n in names[1:]], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t[0])
+        for i, n in enumerate(names[1:]):
+            phase[n] = float(t[i + 1])
+    value = total_ops / (ms * 1e-3)
+
+    # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
+    enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
+    dec_mm, dec_lp = flb.op_cost(priv, "decrypt")
+    enc_lp_launch = enc_lp * CLIENTS * rows
+    achieved = enc_lp_launch / (phase["t_enc"] * 1e-3) / 1e12
+    sm_mhz_max = clk.get("sm_max_mhz") or 1965.0
+    peak = 148 * PEAK_LP_PER_CLK_SM * sm_mhz_max * 1e6 / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json")
+    if os.path.exists(tp):
+        try:
+            with open(tp) as f:
+                traffic = json.load(f).get("dram_bytes_per_launch")
+        except (OSError, ValueError):
+            traffic = None
+
+    # e2e: public API with host buffers (pinned), H2D of the step's inputs and D2H of the result inside
+    e2e = None
+    if not args.no_e2e:
+        pinned_in = [g.pin_memory() for g in grads_host]
+        pinned_out = torch.empty_like(out, device="cpu").pin_memory()
+        dev_in = [torch.empty_like(g) for g in grads]
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for s in range(args.steps):
+            for c in range(CLIENTS):
+                dev_in[c].copy_(pinned_in[c], non_blocking=True)
+            step(2000 + s, gsrc=dev_in)
+            pinned_out.copy_(out, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        e_ms = e0.elapsed_time(e1) / args.steps
+        if world > 1:
+            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t[0])
+        e2e = {"value": total_ops / (e_ms * 1e-3), "unit": UNIT,
+               "h2d_bytes_per_step": CLIENTS * N_VALUES * 4 * world,
+               "d2h_bytes_per_step": N_VALUES * 4 if world == 1 else N_VALUES * 4,
+               "ms_per_step": e_ms, "path": "pinned host gradients -> H2D -> pack/encrypt/reduce/decrypt/unpack -> D2H floats"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cores = cpu_cores()
+        r = oracle_rates(args.cpu_sample_seconds, cores)
+        v, _ = oracle_value(r, rows)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": r["sample"],
+               "per_op_seconds": {"encrypt": r["t_enc"], "decrypt": r["t_dec"], "add": r["t_add"]}}
+
+    launches_per_step = CLIENTS + 1 + 3 + (3 if world > 1 else 0) + 1 + (1 if my_values else 0)
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32-limb bigint (+f64 codec)", "data": "synthetic",
+            "config": {"workload": "C2 Homo-LR aggregation: 2048-bit key, %d clients/GPU x 1,048,576 float32 "
+                                   "values, packed w=32 S=%d (rho=%d, b=%d), encrypt %d, product over clients, "
+                                   "decrypt %d, unpack" % (CLIENTS, S, qbits, pad, CLIENTS * rows * world, rows),
+                       "key_bits": KEY_BITS, "clients_per_gpu": CLIENTS, "values_per_client": N_VALUES,
+                       "plaintexts_per_client": rows, "parallelism": "dp%d (shard by ciphertext)" % world,
+                       "l2": "flushed between steps (256 MiB memset outside the per-step events)"},
+            "breakdown_ms": phase,
+            "ops_per_step": {"encrypt": ops_enc, "decrypt": ops_dec, "add": ops_add},
+            "op_rates": {"encrypt_per_s": ops_enc / (phase["t_enc"] * 1e-3),
+                         "decrypt_per_s": ops_dec / (phase["t_dec"] * 1e-3),
+                         "add_per_s": ops_add / ((phase["t_red"] + phase["t_xchg"]) * 1e-3)},
+            "roofline": {"bound": "alu", "kernel": "k_encrypt<16,8>", "achieved": achieved, "peak": peak,
+                         "unit": "T limb-products/s (IMAD.WIDE.U32 32x32->64, FMA-heavy pipe)",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "per_unit": {"mont_muls": enc_mm, "limb_products": enc_lp},
+                         "peak_basis": "148 SM x 32 IMAD.WIDE/clk/SM x %.0f MHz (guide: IMAD rt=2/SMSP; "
+                                       "IMAD.WIDE half rate, measured tools/imad_peak.cu)" % sm_mhz_max},
+            "decrypt_cost": {"mont_muls": dec_mm, "limb_products": dec_lp},
+            "clocks": clk, "gpu_launches": launches_per_step * args.steps,
+            "e2e": e2e, "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_flb(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -4,6 +4,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -33,7 +34,7 @@ int fail(int code, const std::string& msg) {
     if (e_ != cudaSuccess) return fail(FLB_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
   } while (0)
 
-constexpr int kBlock = 128;
+constexpr int kBlock = 32;  // one warp per block: occupancy follows the register count exactly
 constexpr int kReduceChunk = 64;  // inputs per group in one reduction level
 
 // ----------------------------------------------------------------------------- constant blobs
@@ -452,22 +453,50 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
 }  // namespace
 
 // ----------------------------------------------------------------------------- dispatch macros
-#define FLB_DISPATCH_ENC(frame, FN, ...)                              \
-  switch (frame) {                                                   \
-    case 1024: return FN<16, 4>(__VA_ARGS__);                        \
-    case 2048: return FN<16, 8>(__VA_ARGS__);                        \
-    case 3072: return FN<12, 16>(__VA_ARGS__);                       \
-    case 4096: return FN<16, 16>(__VA_ARGS__);                       \
-    default: return fail(FLB_EUNSUPPORTED, "unsupported key frame"); \
-  }
-#define FLB_DISPATCH_DEC(frame, FN, ...)                              \
-  switch (frame) {                                                   \
-    case 1024: return FN<16, 2>(__VA_ARGS__);                        \
-    case 2048: return FN<16, 4>(__VA_ARGS__);                        \
-    case 3072: return FN<12, 8>(__VA_ARGS__);                        \
-    case 4096: return FN<16, 8>(__VA_ARGS__);                        \
-    default: return fail(FLB_EUNSUPPORTED, "unsupported key frame"); \
-  }
+// Limb split per frame: X limbs per lane, T lanes per big integer.  FLB_LIMBS=8 selects the
+// narrow split (tuning experiments); the default is the wide split.
+static int limbs_per_lane() {
+  static int v = [] {
+    const char* e = getenv("FLB_LIMBS");
+    return (e && atoi(e) == 8) ? 8 : 16;
+  }();
+  return v;
+}
+#define FLB_DISPATCH_ENC(frame, FN, ...)                                           \
+  do {                                                                            \
+    const bool nar = limbs_per_lane() == 8;                                       \
+    switch (frame) {                                                              \
+      case 1024: return nar ? FN<8, 8>(__VA_ARGS__) : FN<16, 4>(__VA_ARGS__);     \
+      case 2048: return nar ? FN<8, 16>(__VA_ARGS__) : FN<16, 8>(__VA_ARGS__);    \
+      case 3072: return FN<12, 16>(__VA_ARGS__);                                  \
+      case 4096: return nar ? FN<8, 32>(__VA_ARGS__) : FN<16, 16>(__VA_ARGS__);   \
+      default: return fail(FLB_EUNSUPPORTED, "unsupported key frame");            \
+    }                                                                             \
+  } while (0)
+#define FLB_DISPATCH_DEC(frame, FN, ...)                                           \
+  do {                                                                            \
+    const bool nar = limbs_per_lane() == 8;                                       \
+    switch (frame) {                                                              \
+      case 1024: return nar ? FN<8, 4>(__VA_ARGS__) : FN<16, 2>(__VA_ARGS__);     \
+      case 2048: return nar ? FN<8, 8>(__VA_ARGS__) : FN<16, 4>(__VA_ARGS__);     \
+      case 3072: return FN<12, 8>(__VA_ARGS__);                                   \
+      case 4096: return nar ? FN<8, 16>(__VA_ARGS__) : FN<16, 8>(__VA_ARGS__);    \
+      default: return fail(FLB_EUNSUPPORTED, "unsupported key frame");            \
+    }                                                                             \
+  } while (0)
+
+namespace {
+template <int X, int T>
+int run_add_plain(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out,
+                  size_t count, cudaStream_t st) {
+  return run_add<X, T, false>(K, dev, a, b, out, count, st);
+}
+template <int X, int T>
+int run_mont_dbg(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out,
+                 size_t count, cudaStream_t st) {
+  return run_add<X, T, true>(K, dev, a, b, out, count, st);
+}
+}  // namespace
 
 extern "C" {
 
@@ -611,15 +640,7 @@ int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* 
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
-#define RUN_ADD(X, T) run_add<X, T, false>(K, dev, c1, c2, out, count, (cudaStream_t)stream)
-  switch (K->frame) {
-    case 1024: return RUN_ADD(16, 4);
-    case 2048: return RUN_ADD(16, 8);
-    case 3072: return RUN_ADD(12, 16);
-    case 4096: return RUN_ADD(16, 16);
-  }
-#undef RUN_ADD
-  return fail(FLB_EUNSUPPORTED, "unsupported key frame");
+  FLB_DISPATCH_ENC(K->frame, run_add_plain, K, dev, c1, c2, out, count, (cudaStream_t)stream);
 }
 
 int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
@@ -629,15 +650,7 @@ int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, u
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
-#define RUN_MONT(X, T) run_add<X, T, true>(K, dev, a, b, out, count, (cudaStream_t)stream)
-  switch (K->frame) {
-    case 1024: return RUN_MONT(16, 4);
-    case 2048: return RUN_MONT(16, 8);
-    case 3072: return RUN_MONT(12, 16);
-    case 4096: return RUN_MONT(16, 16);
-  }
-#undef RUN_MONT
-  return fail(FLB_EUNSUPPORTED, "unsupported key frame");
+  FLB_DISPATCH_ENC(K->frame, run_mont_dbg, K, dev, a, b, out, count, (cudaStream_t)stream);
 }
 
 int flb_scalar_mul(const flb_pub* K, const uint32_t* c, const uint32_t* e, uint32_t e_words, uint32_t* out,

@@ -239,30 +239,80 @@ __device__ __forceinline__ uint32_t collapse(uint32_t (&r)[X], const uint32_t (&
   return ((c >> 1) | (topw != 0)) ? 1u : 0u;
 }
 
-// r = a * b * R^-1 mod N, canonical.  a, b < N (b may be any value < R when a < N).
-// r may alias a or b (all reads of a, b finish before r is written).
+// ----------------------------------------------------------------------------- operand staging
+// The broadcast operand b of a multiplication is staged in shared memory: each CIOS step reads
+// its word b_i with one LDS that every lane of the group hits at the same address (a broadcast),
+// replacing a register-file copy of b plus a shuffle.  Lane k's chunk sits at k*LD with LD = X+4
+// so the 16-byte stores of the T lanes hit distinct bank quads.  Blocks have <= kMaxWarps warps.
+constexpr int kMaxWarps = 4;
+
+template <int X>
+__device__ __forceinline__ uint32_t* stage_base() {
+  constexpr int LD = X + 4;
+  __shared__ __align__(16) uint32_t buf[kMaxWarps * 32 * LD];
+  return buf + (threadIdx.x >> 5) * (32 * LD);
+}
+
+// this group's staging buffer
 template <int X, int T>
-__device__ __forceinline__ void mont_mul(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&b)[X],
-                                         const uint32_t (&n)[X], uint32_t n0inv) {
+__device__ __forceinline__ uint32_t* stage_group() {
+  constexpr int LD = X + 4;
+  return stage_base<X>() + (int)(lane_id() & ~(uint32_t)(T - 1)) * LD;
+}
+
+template <int X, int T>
+__device__ __forceinline__ void stage(const uint32_t (&b)[X]) {
+  constexpr int LD = X + 4;
+  const int k = (int)(lane_id() & (T - 1));
+  uint4* q = reinterpret_cast<uint4*>(stage_group<X, T>() + k * LD);
+  __syncwarp();
+#pragma unroll
+  for (int v = 0; v < X / 4; v++) q[v] = make_uint4(b[4 * v], b[4 * v + 1], b[4 * v + 2], b[4 * v + 3]);
+  __syncwarp();
+}
+
+// r = a * b * R^-1 mod N, canonical, with b staged by stage<X,T>().  a < N (or any a < R when
+// b < N).  r may alias a.
+template <int X, int T>
+__device__ __forceinline__ void mont_mul_staged(uint32_t (&r)[X], const uint32_t (&a)[X],
+                                                const uint32_t (&n)[X], uint32_t n0inv) {
+  constexpr int LD = X + 4;
+  const uint32_t* bs = stage_group<X, T>();
   uint32_t E[X + 1], O[X + 1], pend = 0;
 #pragma unroll
   for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
 #pragma unroll 1
   for (int kk = 0; kk < T; kk++) {
+    const uint32_t* row = bs + kk * LD;
 #pragma unroll
-    for (int jj = 0; jj < X; jj++) {
-      const uint32_t bi = __shfl_sync(FULL, b[jj], kk, T);
-      cios_step<X, T, true>(E, O, pend, a, bi, n, n0inv);
-    }
+    for (int jj = 0; jj < X; jj++) cios_step<X, T, true>(E, O, pend, a, row[jj], n, n0inv);
   }
   const uint32_t over = collapse<X, T>(r, E, O, pend);
   grp_cond_sub<X, T>(r, n, over);
 }
 
+template <int X, int T>
+__device__ __forceinline__ void mont_mul(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&b)[X],
+                                         const uint32_t (&n)[X], uint32_t n0inv) {
+  stage<X, T>(b);
+  mont_mul_staged<X, T>(r, a, n, n0inv);
+}
+
+// r = a * a * R^-1 mod N
+template <int X, int T>
+__device__ __forceinline__ void mont_sqr(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
+                                         uint32_t n0inv) {
+  stage<X, T>(a);
+  mont_mul_staged<X, T>(r, a, n, n0inv);
+}
+
 // r = a * b mod 2^(32*S) (the low half of the plain product).
 template <int X, int T>
 __device__ __forceinline__ void mul_lo(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&b)[X]) {
+  constexpr int LD = X + 4;
   const int k = (int)(lane_id() & (T - 1));
+  stage<X, T>(b);
+  const uint32_t* bs = stage_group<X, T>();
   uint32_t E[X + 1], O[X + 1], pend = 0, res[X];
   const uint32_t dummy_n[X] = {};
 #pragma unroll
@@ -271,10 +321,10 @@ __device__ __forceinline__ void mul_lo(uint32_t (&r)[X], const uint32_t (&a)[X],
   for (int t = 0; t < X; t++) res[t] = 0;
 #pragma unroll 1
   for (int kk = 0; kk < T; kk++) {
+    const uint32_t* row = bs + kk * LD;
 #pragma unroll
     for (int jj = 0; jj < X; jj++) {
-      const uint32_t bi = __shfl_sync(FULL, b[jj], kk, T);
-      const uint32_t w = cios_step<X, T, false>(E, O, pend, a, bi, dummy_n, 0u);
+      const uint32_t w = cios_step<X, T, false>(E, O, pend, a, row[jj], dummy_n, 0u);
       if (k == kk) res[jj] = w;
     }
   }

@@ -9,6 +9,18 @@
 #include <cstdint>
 #include "flb_bn.cuh"
 
+// Launch bounds: one-warp blocks; the minimum resident blocks per SM caps registers per thread
+// (65536 / (32 * MINB)).  Tuned on B200.
+#ifndef FLB_MINB_ENC
+#define FLB_MINB_ENC 14
+#endif
+#ifndef FLB_MINB_DEC
+#define FLB_MINB_DEC 14
+#endif
+#ifndef FLB_MINB_MUL
+#define FLB_MINB_MUL 1
+#endif
+
 namespace flb {
 
 struct ModRef {
@@ -109,7 +121,7 @@ __device__ __forceinline__ void modexp_sched(uint32_t (&acc)[X], uint32_t (&x)[X
   uint32_t b[X];
   store_limbs<X>(tab + k * X, x);
   if (table > 1) {
-    mont_mul<X, T>(b, x, x, n, n0inv);
+    mont_sqr<X, T>(b, x, n, n0inv);
 #pragma unroll 1
     for (int i = 1; i < table; i++) {
       mont_mul<X, T>(x, x, b, n, n0inv);
@@ -127,11 +139,11 @@ __device__ __forceinline__ void modexp_sched(uint32_t (&acc)[X], uint32_t (&x)[X
     for (int i = 0; i < steps; i++) {
       if (i == sq) {
         load_limbs_plain<X>(b, tab + (size_t)idx * stride + k * X);
+        stage<X, T>(b);
       } else {
-#pragma unroll
-        for (int j = 0; j < X; j++) b[j] = acc[j];
+        stage<X, T>(acc);
       }
-      mont_mul<X, T>(acc, acc, b, n, n0inv);
+      mont_mul_staged<X, T>(acc, acc, n, n0inv);
     }
   }
 }
@@ -153,7 +165,7 @@ struct EncArgs {
 
 // c = (1 + m n) r^n mod n^2 (Eq. 3 with g = n+1: g^m = 1 + m n mod n^2).
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_encrypt(const EncArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_ENC) k_encrypt(const EncArgs A) {
   constexpr int S = X * T;
   const Grid<T> g;
   uint32_t n[X];
@@ -204,7 +216,7 @@ struct DecArgs {
 // m = D(c) (Eq. 4) by CRT (reading c10):
 //   m_P = L_P(c^(P-1) mod P^2) h_P mod P, m = m_q + q ((m_p - m_q) q^-1 mod p).
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_decrypt(const DecArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_DEC) k_decrypt(const DecArgs A) {
   constexpr int S = X * T;  // sp
   const Grid<T> g;
   uint32_t* tab = A.scratch + (size_t)g.gid * S;
@@ -264,7 +276,7 @@ struct AddArgs {
 
 // c1 c2 mod n^2 (Eq. 5) = mont(mont(c1, c2), R^2).
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_add(const AddArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_add(const AddArgs A) {
   constexpr int S = X * T;
   const Grid<T> g;
   uint32_t n[X];
@@ -286,7 +298,7 @@ __global__ void __launch_bounds__(128) k_add(const AddArgs A) {
 
 // ----------------------------------------------------------------------------- debug mont_mul
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_mont(const AddArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_mont(const AddArgs A) {
   constexpr int S = X * T;
   const Grid<T> g;
   uint32_t n[X];
@@ -326,7 +338,7 @@ __device__ __forceinline__ uint32_t exp_window(const uint32_t* e, uint32_t e_wor
 // c^e mod n^2 (mod_pow; reading c19), per-element exponent, fixed window with
 // an always-multiply step (table[0] = Montgomery one) so control flow is uniform.
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_scalar_mul(const SmulArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_ENC) k_scalar_mul(const SmulArgs A) {
   constexpr int S = X * T;
   const Grid<T> g;
   uint32_t n[X];
@@ -366,11 +378,7 @@ __global__ void __launch_bounds__(128) k_scalar_mul(const SmulArgs A) {
     for (int w = top; w >= 0; w--) {
       if (w != top) {
 #pragma unroll 1
-        for (int s = 0; s < A.bw; s++) {
-#pragma unroll
-          for (int j = 0; j < X; j++) b[j] = acc[j];
-          mont_mul<X, T>(acc, acc, b, n, n0inv);
-        }
+        for (int s = 0; s < A.bw; s++) mont_sqr<X, T>(acc, acc, n, n0inv);
       }
       const uint32_t d = valid ? exp_window(ep, A.e_words, w, A.bw) : 0u;
       load_limbs_plain<X>(b, tab + (size_t)d * stride + g.k * X);
@@ -400,7 +408,7 @@ struct RedArgs {
 // raw-input Montgomery products it is prod * R^-(L-1); one product with R^L mod n^2 removes the
 // factor.  Lanes whose chunk is shorter multiply by R mod n^2 (a no-op).
 template <int X, int T>
-__global__ void __launch_bounds__(128) k_reduce(const RedArgs A) {
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_reduce(const RedArgs A) {
   constexpr int S = X * T;
   const Grid<T> g;
   uint32_t n[X];

@@ -1,0 +1,146 @@
+"""CPU tests of the C ABI: the library loads, exports every symbol include/flb_paillier.h declares,
+and its host-side logic (key import/generation/export, argument validation, cost accounting)
+behaves — no device work is launched here."""
+
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_icde_zeng0fcpcwg23_b200 as flb
+from paper_conf_icde_zeng0fcpcwg23_b200 import _lib
+from tests.helpers import golden_keys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "flb_paillier.h")
+KEYS = golden_keys()
+
+
+def declared_symbols():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(flb_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_header_declares_the_boundary():
+    syms = declared_symbols()
+    for s in ["flb_keygen", "flb_key_from_primes", "flb_encrypt", "flb_decrypt", "flb_add", "flb_scalar_mul",
+              "flb_reduce_segments", "flb_pack", "flb_unpack", "flb_unpack_sums", "flb_last_error"]:
+        assert s in syms
+
+
+def test_library_exports_every_declared_symbol():
+    out = subprocess.run(["nm", "-D", "--defined-only", _lib.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (flb_[a-z0-9_]+)\b", out))
+    missing = [s for s in declared_symbols() if s not in exported]
+    assert not missing, missing
+    # and the binding binds exactly the declared set
+    assert sorted(_lib.SIGNATURES) == declared_symbols()
+    lib = ctypes.CDLL(_lib.LIB_PATH)
+    for s in declared_symbols():
+        getattr(lib, s)
+
+
+def test_library_is_sm100a():
+    out = subprocess.run(["cuobjdump", "--list-elf", _lib.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+@pytest.mark.parametrize("name,bits,ptw,ctw", [("toy9", 9, 32, 64), ("toy16", 16, 32, 64), ("1024", 1024, 32, 64),
+                                               ("2048", 2048, 64, 128), ("3072", 3072, 96, 192),
+                                               ("4096", 4096, 128, 256)])
+def test_key_import_export(name, bits, ptw, ctw):
+    p, q = KEYS[name]
+    pub, priv = flb.key_from_primes(q, p)  # order does not matter; p becomes the larger
+    assert (pub.bits, pub.pt_words, pub.ct_words) == (bits, ptw, ctw)
+    P, Q, N = priv.export()
+    assert (P, Q, N) == (max(p, q), min(p, q), p * q)
+    assert pub.slot_capacity(32) == (bits - 1) // 32
+
+
+def test_keygen_deterministic_and_valid():
+    pub, priv = flb.keygen(1024, 12345)
+    p, q, n = priv.export()
+    pub2, priv2 = flb.keygen(1024, 12345)
+    assert priv2.export() == (p, q, n)
+    assert flb.keygen(1024, 12346)[1].export() != (p, q, n)
+    assert n.bit_length() == 1024 and p.bit_length() == q.bit_length() == 512
+    for x in (p, q):  # independent check: Fermat + small trial division
+        assert all(pow(b, x - 1, x) == 1 for b in (2, 3, 5, 7, 11))
+        assert all(x % d for d in range(3, 2000, 2))
+
+
+@pytest.mark.parametrize("p,q,code", [(251, 251, -4), (251, 255, -4), (250, 241, -4), (1, 241, -4),
+                                      (7, 3, -4)])  # gcd(21, 12) = 3
+def test_key_import_rejects(p, q, code):
+    with pytest.raises(flb.FlbError) as e:
+        flb.key_from_primes(p, q)
+    assert e.value.code == code
+
+
+def test_key_import_rejects_oversize():
+    p = (1 << 2100) + 1  # size check happens before primality
+    with pytest.raises(flb.FlbError) as e:
+        flb.key_from_primes(p, p + 2)
+    assert e.value.code == -5
+
+
+def test_keygen_rejects_bad_size():
+    with pytest.raises(flb.FlbError) as e:
+        flb.keygen(1000, 1)
+    assert e.value.code == -1
+
+
+def test_batch_calls_validate_before_launch():
+    p, q = KEYS["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    L = _lib.LIB
+    assert L.flb_encrypt(pub.handle, None, None, 0, 0, None, 4, None) == -1
+    assert L.flb_decrypt(priv.handle, None, None, 4, None) == -1
+    assert L.flb_add(pub.handle, None, None, None, 4, None) == -1
+    assert L.flb_scalar_mul(pub.handle, 16, 16, 0, 16, 4, None) == -1  # e_words = 0
+    assert L.flb_reduce_segments(pub.handle, None, 3, None, None, 2, 0, None, None) == -1
+    assert "null" in L.flb_last_error().decode()
+    # count = 0 is a no-op that needs no device
+    assert L.flb_encrypt(pub.handle, 16, None, 0, 0, 16, 0, None) == 0
+    bad = [(1.0, 29, 3, 32, 32), (1.0, 29, 4, 33, 1), (0.0, 29, 3, 32, 1), (1.0, 53, 11, 64, 1), (1.0, 29, 3, 32, 0)]
+    for a, qb, pb, sb, sl in bad:
+        cs = _lib.CodecStruct(a, qb, pb, sb, sl)
+        assert L.flb_pack(pub.handle, ctypes.byref(cs), 16, 10, 16, None) == -1
+        assert L.flb_unpack(pub.handle, ctypes.byref(cs), 16, 10, None, 1, 16, None) == -1
+
+
+def _sliding_mults(e, w):
+    """Independent count of a left-to-right odd-power sliding window (table + squarings + products)."""
+    bits = bin(e)[2:]
+    table = 1 << (w - 1)
+    cost = table if table > 1 else 0
+    i, first = 0, True
+    while i < len(bits):
+        if bits[i] == "0":
+            cost += 1
+            i += 1
+            continue
+        j = min(len(bits), i + w)
+        while bits[j - 1] == "0":
+            j -= 1
+        cost += 0 if first else (j - i) + 1
+        first = False
+        i = j
+    return cost
+
+
+def test_op_cost_matches_independent_window_count():
+    p, q = KEYS["2048"]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    mm, lp = flb.op_cost(pub, "encrypt")
+    best = min(_sliding_mults(n, w) for w in range(1, 8))
+    assert mm == best + 3  # + to-Montgomery, m*n, final product
+    assert lp == mm * (2 * 128 * 128 + 128)
+    mm_d, lp_d = flb.op_cost(priv, "decrypt")
+    bd = sum(min(_sliding_mults(P - 1, w) for w in range(1, 8)) for P in (p, q))
+    assert mm_d == bd + 2 * 4 + 2
+    assert flb.op_cost(pub, "add") == (2, 2 * (2 * 128 * 128 + 128))
