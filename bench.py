@@ -237,9 +237,13 @@ def run_flb(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    backend = os.environ.get("FLB_DIST_BACKEND", "nccl")  # gloo: multi-rank logic check on one GPU
     if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        torch.cuda.set_device(local % torch.cuda.device_count())
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     else:
         torch.cuda.set_device(0)
     dev = torch.device("cuda", torch.cuda.current_device())
@@ -313,7 +317,7 @@ def run_flb(args):
     torch.cuda.synchronize()
     ev.clear()
 
-    clocks = ClockSampler(torch.cuda.current_device() if world == 1 else local)
+    clocks = ClockSampler(torch.cuda.current_device())
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -335,7 +339,8 @@ def run_flb(args):
             phase[b] += ev[a][s].elapsed_time(ev[b][s]) / args.steps
     ms = sum(step_ms) / len(step_ms)
     if world > 1:
-        t = torch.tensor([ms] + [phase[n] for n in names[1:]], dtype=torch.float64, device=dev)
+        t = torch.tensor([ms] + [phase[n] for n in names[1:]], dtype=torch.float64,
+                         device=dev if backend == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t[0])
         for i, n in enumerate(names[1:]):
@@ -379,7 +384,7 @@ def run_flb(args):
         torch.cuda.synchronize()
         e_ms = e0.elapsed_time(e1) / args.steps
         if world > 1:
-            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+            t = torch.tensor([e_ms], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_ms = float(t[0])
         e2e = {"value": total_ops / (e_ms * 1e-3), "unit": UNIT,

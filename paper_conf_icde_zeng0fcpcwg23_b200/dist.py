@@ -60,7 +60,13 @@ def exchange_and_finish(partial: torch.Tensor, group, reduce: Callable, world: i
     rpr = rows_p // world
     if recv is None:
         recv = torch.empty_like(partial)
-    dist.all_to_all_single(recv, partial, group=group)
+    if partial.is_cuda and dist.get_backend(group) == "gloo":
+        # gloo has no CUDA all_to_all: stage through host memory (CPU tests / single-GPU multi-rank runs)
+        host = torch.empty_like(partial, device="cpu")
+        dist.all_to_all_single(host, partial.cpu(), group=group)
+        recv.copy_(host)
+    else:
+        dist.all_to_all_single(recv, partial, group=group)
     offsets, idx = finish_segments(world, rpr, device=partial.device)
     return reduce(recv, offsets, idx, world)
 
