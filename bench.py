@@ -50,6 +50,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-sample-seconds", type=float, default=20.0)
+    ap.add_argument("--encrypt", choices=["keyholder", "public"], default="keyholder",
+                    help="C2 clients hold the key pair (they decrypt the aggregate, Fig. 2), so they may "
+                         "encrypt by CRT; 'public' uses the public-key-only kernel")
     return ap.parse_args()
 
 
@@ -293,7 +296,10 @@ def run_flb(args):
         for c in range(CLIENTS):
             flb.pack(pub, cd, grads[c] if gsrc is None else gsrc[c], out=pt[c * rows:(c + 1) * rows])
         mark("t_pack")
-        flb.encrypt(pub, pt, seed=seed, ctr0=rank * CLIENTS * rows, out=ct)
+        if args.encrypt == "keyholder":
+            flb.encrypt_crt(priv, pt, seed=seed, ctr0=rank * CLIENTS * rows, out=ct)
+        else:
+            flb.encrypt(pub, pt, seed=seed, ctr0=rank * CLIENTS * rows, out=ct)
         mark("t_enc")
         flb.reduce_segments(pub, ct, offs, idx=idx, max_segment_len=CLIENTS, out=part)
         mark("t_red")
@@ -347,15 +353,33 @@ def run_flb(args):
             phase[n] = float(t[i + 1])
     value = total_ops / (ms * 1e-3)
 
+    # the other encryption path, timed once on the same batch (reported, not part of the step)
+    other = "public" if args.encrypt == "keyholder" else "keyholder"
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    if other == "public":
+        flb.encrypt(pub, pt, seed=7, out=ct)
+    else:
+        flb.encrypt_crt(priv, pt, seed=7, out=ct)
+    e1.record()
+    torch.cuda.synchronize()
+    other_rate = ops_enc / world / (e0.elapsed_time(e1) * 1e-3)
+
     # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
-    enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
+    if args.encrypt == "keyholder":
+        enc_mm, enc_lp = flb.op_cost(priv, "encrypt_crt")
+        enc_kernel = "k_encrypt_crt<16,4>"
+    else:
+        enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
+        enc_kernel = "k_encrypt<16,8>"
     dec_mm, dec_lp = flb.op_cost(priv, "decrypt")
     enc_lp_launch = enc_lp * CLIENTS * rows
     achieved = enc_lp_launch / (phase["t_enc"] * 1e-3) / 1e12
     sm_mhz_max = clk.get("sm_max_mhz") or 1965.0
     peak = 148 * PEAK_LP_PER_CLK_SM * sm_mhz_max * 1e6 / 1e12
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json")
+    tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json" if args.encrypt == "public" else
+                      "encrypt_crt_traffic.json")
     if os.path.exists(tp):
         try:
             with open(tp) as f:
@@ -407,8 +431,9 @@ def run_flb(args):
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32-limb bigint (+f64 codec)", "data": "synthetic",
             "config": {"workload": "C2 Homo-LR aggregation: 2048-bit key, %d clients/GPU x 1,048,576 float32 "
-                                   "values, packed w=32 S=%d (rho=%d, b=%d), encrypt %d, product over clients, "
-                                   "decrypt %d, unpack" % (CLIENTS, S, qbits, pad, CLIENTS * rows * world, rows),
+                                   "values, packed w=32 S=%d (rho=%d, b=%d), encrypt %d (%s), product over "
+                                   "clients, decrypt %d, unpack" % (CLIENTS, S, qbits, pad, CLIENTS * rows * world,
+                                                                    args.encrypt, rows),
                        "key_bits": KEY_BITS, "clients_per_gpu": CLIENTS, "values_per_client": N_VALUES,
                        "plaintexts_per_client": rows, "parallelism": "dp%d (shard by ciphertext)" % world,
                        "l2": "flushed between steps (256 MiB memset outside the per-step events)"},
@@ -416,8 +441,11 @@ def run_flb(args):
             "ops_per_step": {"encrypt": ops_enc, "decrypt": ops_dec, "add": ops_add},
             "op_rates": {"encrypt_per_s": ops_enc / (phase["t_enc"] * 1e-3),
                          "decrypt_per_s": ops_dec / (phase["t_dec"] * 1e-3),
-                         "add_per_s": ops_add / ((phase["t_red"] + phase["t_xchg"]) * 1e-3)},
-            "roofline": {"bound": "alu", "kernel": "k_encrypt<16,8>", "achieved": achieved, "peak": peak,
+                         "add_per_s": ops_add / ((phase["t_red"] + phase["t_xchg"]) * 1e-3),
+                         ("encrypt_public_per_gpu_per_s" if other == "public" else "encrypt_keyholder_per_gpu_per_s"):
+                             other_rate},
+            "encrypt_mode": args.encrypt,
+            "roofline": {"bound": "alu", "kernel": enc_kernel, "achieved": achieved, "peak": peak,
                          "unit": "T limb-products/s (IMAD.WIDE.U32 32x32->64, FMA-heavy pipe)",
                          "frac": achieved / peak, "traffic": traffic,
                          "per_unit": {"mont_muls": enc_mm, "limb_products": enc_lp},

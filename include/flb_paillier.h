@@ -88,6 +88,14 @@ uint32_t flb_slot_capacity(const flb_pub* pub, uint32_t slot_bits);
 int flb_encrypt(const flb_pub* pub, const uint32_t* m, const uint32_t* r, uint64_t seed,
                 uint64_t ctr0, uint32_t* c, size_t count, void* stream);
 
+/* Encryption by a holder of the private key: the same c_i as flb_encrypt (same m, r, seed,
+ * ctr0 -> the same bits), computed as (1 + m n) r^n mod p^2 and mod q^2 with half-size moduli and
+ * recombined by CRT (c = c_q + q^2 ((c_p - c_q) (q^2)^-1 mod p^2)) — about half the limb products.
+ * Beyond the paper; in Fig. 2 the clients that encrypt also
+ * decrypt, so they hold the key.  Arguments and errors as flb_encrypt. */
+int flb_encrypt_crt(const flb_priv* priv, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                    uint64_t ctr0, uint32_t* c, size_t count, void* stream);
+
 /* Paillier::decrypt (Eq. 4), by CRT (reading c10).  c: [count][ct_words]
  * (each a unit < n^2), m: [count][pt_words] receives m_i in [0, n).  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_decrypt(const flb_priv* priv, const uint32_t* c, uint32_t* m, size_t count, void* stream);
@@ -148,7 +156,8 @@ int flb_debug_mont_mul(const flb_pub* pub, const uint32_t* a, const uint32_t* b,
  * multiplications the kernel performs per element (window table, schedule, domain entry/exit),
  * *limb_products = their CIOS limb-product count (2s^2 + s per s-limb multiplication, s^2 for
  * the plain low-half product of the exact division).  op: 0 = encrypt (pub), 1 = decrypt
- * (priv), 2 = add (pub), 3 = one reduce input (pub; excludes the per-chunk fix-up).
+ * (priv), 2 = add (pub), 3 = one reduce input (pub; excludes the per-chunk fix-up),
+ * 4 = key-holder encrypt (priv).
  * Host only.  Errors: FLB_EINVAL. */
 int flb_op_cost(const flb_pub* pub, const flb_priv* priv, int op, uint64_t* mont_muls,
                 uint64_t* limb_products);

@@ -20,7 +20,7 @@ from . import _lib
 from ._lib import LIB, FlbError, check
 
 __all__ = [
-    "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "decrypt", "add",
+    "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
     "Codec", "FlbError", "library_path", "op_cost",
 ]
@@ -134,6 +134,21 @@ def encrypt(pub: PublicKey, m: torch.Tensor, r: Optional[torch.Tensor] = None, s
     _check_batch(out, pub.ct_words, "out")
     check("flb_encrypt", LIB.flb_encrypt(pub.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0, _ptr(out), M,
                                          _stream(stream)))
+    return out
+
+
+def encrypt_crt(priv: PrivateKey, m: torch.Tensor, r: Optional[torch.Tensor] = None, seed: int = 0, ctr0: int = 0,
+                out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """Key-holder encryption: the same ciphertexts as ``encrypt`` via CRT over p^2, q^2 (~2x fewer limb products)."""
+    pub = priv.pub
+    M = _check_batch(m, pub.pt_words, "m")
+    if r is not None:
+        _check_batch(r, pub.pt_words, "r")
+    if out is None:
+        out = torch.empty((M, pub.ct_words), dtype=torch.int32, device=m.device)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_encrypt_crt", LIB.flb_encrypt_crt(priv.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0,
+                                                 _ptr(out), M, _stream(stream)))
     return out
 
 
@@ -251,7 +266,7 @@ def unpack_sums(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int, o
     return out
 
 
-OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3}
+OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3, "encrypt_crt": 4}
 
 
 def op_cost(key, op: str) -> Tuple[int, int]:

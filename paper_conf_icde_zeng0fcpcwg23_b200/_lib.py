@@ -45,6 +45,7 @@ SIGNATURES = {
     "flb_ct_words": (_U32, [_P]),
     "flb_slot_capacity": (_U32, [_P, _U32]),
     "flb_encrypt": (ctypes.c_int, [_P, _P, _P, _U64, _U64, _P, _SZ, _P]),
+    "flb_encrypt_crt": (ctypes.c_int, [_P, _P, _P, _U64, _U64, _P, _SZ, _P]),
     "flb_decrypt": (ctypes.c_int, [_P, _P, _P, _SZ, _P]),
     "flb_add": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
     "flb_scalar_mul": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),

@@ -115,8 +115,10 @@ struct flb_priv {
     uint32_t P_n0inv, P2_n0inv;
     H::Schedule sched;
     size_t o_P, o_P2, o_R2, o_R3, o_Pinv, o_hR, o_sched;
+    size_t o_nR;  // n R mod P^2 (key-holder encryption)
   } pr[2];
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
+  size_t o_q2invR = 0, o_enc_sched = 0;  // key-holder encryption: (q^2)^-1 R mod p^2, schedule of n
   uint32_t n_n0inv = 0;
   Blob blob;
   DevBlob dev;
@@ -188,6 +190,19 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
     R.o_Pinv = V->blob.put(H::inv_mod_2k(P, sp), sp);
     R.o_hR = V->blob.put(C1.to(h), sp);
     R.o_sched = V->blob.put_raw(R.sched.ops);
+    R.o_nR = V->blob.put(C2.to(H::mod(V->pub->n, R.P2)), sp);
+  }
+  {
+    // (q^2)^-1 mod p^2 by Euler: a^(phi(p^2) - 1), phi(p^2) = p (p - 1)
+    H::MontCtx Cp2(V->pr[0].P2);
+    Limbs phi = H::resized(H::mul(V->p, [&] { Limbs t = V->p; H::sub_in(t, one); return t; }()), 2 * sp);
+    Limbs e = phi;
+    Limbs one2(e.size(), 0);
+    one2[0] = 1;
+    H::sub_in(e, one2);
+    const Limbs q2inv = Cp2.pow(H::mod(V->pr[1].P2, V->pr[0].P2), e);
+    V->o_q2invR = V->blob.put(Cp2.to(q2inv), sp);
+    V->o_enc_sched = V->blob.put_raw(V->pub->enc.ops);
   }
   // CRT recombination constants
   H::MontCtx Cn(V->pub->n), Cp(V->p);
@@ -328,6 +343,41 @@ int run_decrypt(const flb_priv* V, const uint32_t* dev, const uint32_t* c, uint3
   A.count = count;
   A.scratch = (uint32_t*)sc.p;
   flb::k_decrypt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_encrypt_crt(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                    uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt_crt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const flb_pub* K = V->pub;
+  Scratch sc;
+  rc = sc.alloc((size_t)K->enc.table * G * K->sp * 4, st);
+  if (rc) return rc;
+  flb::EncCrtArgs A;
+  for (int i = 0; i < 2; i++) {
+    A.P2[i] = {dev + V->pr[i].o_P2, V->pr[i].P2_n0inv};
+    A.R2[i] = dev + V->pr[i].o_R2;
+    A.nR[i] = dev + V->pr[i].o_nR;
+  }
+  A.q2 = dev + V->pr[1].o_P2;
+  A.q2invR = dev + V->o_q2invR;
+  A.sched = dev + V->o_enc_sched;
+  A.sched_len = (int)K->enc.ops.size();
+  A.table = K->enc.table;
+  A.nbits = K->nbits;
+  A.m = m;
+  A.r = r;
+  A.c = c;
+  A.count = count;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt_crt<X, T><<<grid, kBlock, 0, st>>>(A);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }
@@ -531,6 +581,12 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       *limb_products = mm * csp + lp;
       return FLB_OK;
     }
+    case 4: {  // key-holder encryption: per prime 1 + table + schedule + 2 at sp; CRT 1 + plain product
+      const uint64_t per = 1 + sched_mults(P->enc) + 2;
+      *mont_muls = 2 * per + 1;
+      *limb_products = (2 * per + 1) * csp + sp * sp;
+      return FLB_OK;
+    }
     case 2:
       *mont_muls = 2;
       *limb_products = 2 * cs;
@@ -632,6 +688,16 @@ int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count,
   int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
   if (rc) return rc;
   FLB_DISPATCH_DEC(V->pub->frame, run_decrypt, V, dev, c, m, count, (cudaStream_t)stream);
+}
+
+int flb_encrypt_crt(const flb_priv* V, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0,
+                    uint32_t* c, size_t count, void* stream) {
+  if (!V || !m || !c) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt, V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 
 int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* out, size_t count, void* stream) {

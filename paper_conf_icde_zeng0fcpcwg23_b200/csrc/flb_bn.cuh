@@ -332,6 +332,34 @@ __device__ __forceinline__ void mul_lo(uint32_t (&r)[X], const uint32_t (&a)[X],
   for (int t = 0; t < X; t++) r[t] = res[t];
 }
 
+// (lo, hi) = a * b, the full 2S-limb plain product (hi < R since a, b < R).
+template <int X, int T>
+__device__ __forceinline__ void mul_full(uint32_t (&lo)[X], uint32_t (&hi)[X], const uint32_t (&a)[X],
+                                         const uint32_t (&b)[X]) {
+  constexpr int LD = X + 4;
+  const int k = (int)(lane_id() & (T - 1));
+  stage<X, T>(b);
+  const uint32_t* bs = stage_group<X, T>();
+  uint32_t E[X + 1], O[X + 1], pend = 0, res[X];
+  const uint32_t dummy_n[X] = {};
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
+#pragma unroll
+  for (int t = 0; t < X; t++) res[t] = 0;
+#pragma unroll 1
+  for (int kk = 0; kk < T; kk++) {
+    const uint32_t* row = bs + kk * LD;
+#pragma unroll
+    for (int jj = 0; jj < X; jj++) {
+      const uint32_t w = cios_step<X, T, false>(E, O, pend, a, row[jj], dummy_n, 0u);
+      if (k == kk) res[jj] = w;
+    }
+  }
+#pragma unroll
+  for (int t = 0; t < X; t++) lo[t] = res[t];
+  collapse<X, T>(hi, E, O, pend);
+}
+
 // ----------------------------------------------------------------------------- loads / stores
 template <int X>
 __device__ __forceinline__ void load_limbs(uint32_t (&r)[X], const uint32_t* __restrict__ p) {

@@ -246,7 +246,12 @@ __global__ void __launch_bounds__(32, FLB_MINB_DEC) k_decrypt(const DecArgs A) {
       mul_lo<X, T>(hi, lo, b);                            // L = (x - 1) / P (exact division)
       load_mod<X, T>(n, pa.P);
       load_const<X, T>(b, pa.hR);
-      mont_mul<X, T>(mres[P], hi, b, n, pa.P.n0inv);      // m_P = L h_P mod P
+      mont_mul<X, T>(x, hi, b, n, pa.P.n0inv);            // m_P = L h_P mod P
+#pragma unroll
+      for (int j = 0; j < X; j++) {
+        if (P == 0) mres[0][j] = x[j];
+        else mres[1][j] = x[j];
+      }
     }
     uint32_t n[X], d[X], t[X];
     load_mod<X, T>(n, A.pr[0].P);
@@ -261,6 +266,78 @@ __global__ void __launch_bounds__(32, FLB_MINB_DEC) k_decrypt(const DecArgs A) {
     mont_mul<X, T>(d, d, t, n, A.n.n0inv);                     // q u (< n, exact)
     grp_add<X, T>(d, d, mres[1]);                              // m = m_q + q u
     if (valid) store_limbs<X>(A.m + e * S + g.k * X, d);
+  }
+}
+
+// ----------------------------------------------------------------------------- key-holder encrypt
+struct EncCrtArgs {
+  ModRef P2[2];            // p^2, q^2 in the sp frame
+  const uint32_t* R2[2];   // R^2 mod P^2
+  const uint32_t* nR[2];   // n R mod P^2
+  const uint32_t* q2;      // q^2 (sp limbs, plain)
+  const uint32_t* q2invR;  // (q^2)^-1 R mod p^2
+  const uint32_t* sched;   // schedule of the exponent n (same as the public path)
+  int sched_len, table;
+  uint32_t nbits;
+  const uint32_t* m;       // [count][sp]
+  const uint32_t* r;       // [count][sp] or null (Philox)
+  uint32_t* c;             // [count][2 sp]
+  uint64_t count, seed, ctr0;
+  uint32_t* scratch;       // table * G * sp
+};
+
+// Same bits as k_encrypt (Eq. 3, g = n+1) for a party holding p, q:
+//   c_P = (1 + m n) r^n mod P^2 for P in {p, q} (sp-limb moduli, exponent n itself, so every r
+//   gives the public-path value), then c = c_q + q^2 ((c_p - c_q) (q^2)^-1 mod p^2) < n^2.
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_DEC) k_encrypt_crt(const EncCrtArgs A) {
+  constexpr int S = X * T;  // sp
+  const Grid<T> g;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t cres[2][X];
+#pragma unroll 1
+    for (int P = 0; P < 2; P++) {
+      uint32_t n[X], x[X], b[X], acc[X];
+      load_mod<X, T>(n, A.P2[P]);
+      const uint32_t n0inv = A.P2[P].n0inv;
+      if (A.r) load_elem<X, T>(x, A.r + e * S, S, valid);
+      else philox_r<X, T>(x, A.seed, A.ctr0 + e, S, A.nbits);
+      load_const<X, T>(b, A.R2[P]);
+      mont_mul<X, T>(x, x, b, n, n0inv);                       // r R mod P^2
+      modexp_sched<X, T>(acc, x, A.sched, A.sched_len, A.table, tab, stride, n, n0inv);  // r^n R
+      load_elem<X, T>(x, A.m + e * S, S, valid);
+      load_const<X, T>(b, A.nR[P]);
+      mont_mul<X, T>(x, x, b, n, n0inv);                       // m n mod P^2
+      set_one<X, T>(b);
+      const uint32_t cy = grp_add<X, T>(x, x, b);
+      grp_cond_sub<X, T>(x, n, cy);                            // 1 + m n mod P^2
+      mont_mul<X, T>(acc, acc, x, n, n0inv);                   // c_P
+#pragma unroll
+      for (int j = 0; j < X; j++) {
+        if (P == 0) cres[0][j] = acc[j];
+        else cres[1][j] = acc[j];
+      }
+    }
+    uint32_t n[X], d[X], t[X], hi[X];
+    load_mod<X, T>(n, A.P2[0]);
+    const uint32_t br = grp_sub<X, T>(d, cres[0], cres[1]);   // c_p - c_q (c_q < q^2 < p^2)
+#pragma unroll
+    for (int j = 0; j < X; j++) t[j] = br ? n[j] : 0u;
+    grp_add<X, T>(d, d, t);                                    // mod p^2
+    load_const<X, T>(t, A.q2invR);
+    mont_mul<X, T>(d, d, t, n, A.P2[0].n0inv);                 // u = (c_p - c_q) q^-2 mod p^2
+    load_const<X, T>(t, A.q2);
+    mul_full<X, T>(d, hi, d, t);                               // q^2 u (2 sp limbs)
+    const uint32_t cy = grp_add<X, T>(d, d, cres[1]);          // + c_q
+    grp_add_small<X, T>(hi, cy);
+    if (valid) {
+      store_limbs<X>(A.c + e * (2 * S) + g.k * X, d);
+      store_limbs<X>(A.c + e * (2 * S) + S + g.k * X, hi);
+    }
   }
 }
 

@@ -99,6 +99,38 @@ def test_encrypt_philox_r(name):
         assert got[i] == paillier.encrypt(n, m[i], r), i
 
 
+@pytest.mark.parametrize("name", ALL)
+def test_encrypt_crt_matches_oracle(name):
+    """Key-holder CRT encryption gives exactly Eq. 3's value, for caller and Philox r (any r)."""
+    pub, priv, p, q = key(name)
+    n = p * q
+    cnt = COUNT[name]
+    m = rand_below(n, cnt, 14)
+    r = [x if x else 1 for x in rand_below(n, cnt, 15)]
+    m[0], m[-1] = 0, n - 1
+    r[1] = p if p < n else 1          # r sharing a factor with n: still the public-path value
+    got = from_dev(flb.encrypt_crt(priv, to_dev(m, pub.pt_words), r=to_dev(r, pub.pt_words)))
+    for i in range(cnt):
+        assert got[i] == paillier.encrypt(n, m[i], r[i]), i
+    seed, ctr0 = 0xFEDCBA9876543210, 77
+    got = from_dev(flb.encrypt_crt(priv, to_dev(m, pub.pt_words), seed=seed, ctr0=ctr0))
+    for i in range(cnt):
+        assert got[i] == paillier.encrypt(n, m[i], philox.draw_r(n, seed, ctr0 + i, pub.pt_words)), i
+
+
+def test_encrypt_crt_equals_public_path_at_scale():
+    pub, priv, p, q = key("2048")
+    n = p * q
+    M = 3000
+    m = to_dev(rand_below(n, M, 16), pub.pt_words)
+    a = flb.encrypt(pub, m, seed=5, ctr0=9)
+    b = flb.encrypt_crt(priv, m, seed=5, ctr0=9)
+    assert torch.equal(a, b)
+    got = from_dev(b)
+    for i in (0, 1, 1234, M - 1):
+        assert got[i] == paillier.encrypt(n, from_dev(m[i:i + 1])[0], philox.draw_r(n, 5, 9 + i, pub.pt_words))
+
+
 # ----------------------------------------------------------------------------- decrypt
 
 @pytest.mark.parametrize("name", ALL)

@@ -16,7 +16,7 @@ if [ "${NCU:-1}" = "1" ]; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
     --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e \
     > gpurun_out/${TAG}_bench_under_ncu.log 2>&1
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"k_encrypt" -c 1 \
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"k_encrypt" -c 2 \
     -o gpurun_out/${TAG}_prof_enc python tools/prof_c2.py > gpurun_out/${TAG}_ncu_full.log 2>&1
 fi
 cat gpurun_out/${TAG}_pytest_gpu.txt gpurun_out/${TAG}_smoke.txt

@@ -16,6 +16,7 @@ cd = flb.Codec(1.0, 29, 3, 63)
 rows = cd.num_plaintexts(1 << 20)
 pt = torch.cat([flb.pack(pub, cd, torch.from_numpy(synthetic.c2_gradient(c)).cuda()) for c in range(clients)])
 ct = flb.encrypt(pub, pt, seed=1)
+ct2 = flb.encrypt_crt(priv, pt, seed=1)
 offs, idx = fdist.client_segments(clients, rows, device="cuda")
 agg = flb.reduce_segments(pub, ct, offs, idx=idx, max_segment_len=clients)
 dec = flb.decrypt(priv, agg)

@@ -40,6 +40,13 @@ mm, lp = flb.op_cost(pub, "encrypt")
 res["enc_ms"] = t
 res["enc_per_s"] = M / t * 1e3
 res["enc_TLPs"] = lp * M / t / 1e9
+c2 = torch.empty_like(c)
+t = timed(lambda: flb.encrypt_crt(priv, m, seed=1, out=c2))
+mm, lp = flb.op_cost(priv, "encrypt_crt")
+res["enc_crt_ms"] = t
+res["enc_crt_per_s"] = M / t * 1e3
+res["enc_crt_TLPs"] = lp * M / t / 1e9
+res["enc_crt_equal"] = bool(torch.equal(c, c2))
 Md = min(M, int(os.environ.get("MD", str(M))))
 d = flb.decrypt(priv, c[:Md])
 t = timed(lambda: flb.decrypt(priv, c[:Md], out=d))
