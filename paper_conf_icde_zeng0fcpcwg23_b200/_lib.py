@@ -11,7 +11,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.environ.get("FLB_LIB_PATH", os.path.join(_HERE, "_flb.so"))
+LIB_PATH = os.environ.get("FLB_LIB_PATH") or os.path.join(_HERE, "_flb.so")
 
 FLB_OK = 0
 ERRORS = {-1: "FLB_EINVAL", -2: "FLB_ENOMEM", -3: "FLB_ECUDA", -4: "FLB_EKEY", -5: "FLB_EUNSUPPORTED"}

@@ -13,7 +13,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.environ.get("FLB_LIB_PATH", os.path.join(HERE, "_flb.so"))
+OUT = os.environ.get("FLB_LIB_PATH") or os.path.join(HERE, "_flb.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 FLAGS = [

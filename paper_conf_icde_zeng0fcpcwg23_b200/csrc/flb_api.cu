@@ -251,14 +251,34 @@ int resident_blocks(K kernel, int* blocks) {
   return FLB_OK;
 }
 
-// grid for `items` work units of T lanes each, capped at the resident capacity
+// Grid for `items` work units of T lanes each: at most the resident capacity; the units are then
+// spread evenly over the rounds the persistent loop needs (ceil(items / capacity)), so the last
+// round is not a sliver of the grid — only with FLB_BALANCE=1: measured slower on B200 (fewer
+// resident warps cost more than the partial last round).
+static bool balance_rounds() {
+  static bool v = [] {
+    const char* e = getenv("FLB_BALANCE");
+    return e && atoi(e) == 1;
+  }();
+  return v;
+}
+
 template <int T, typename K>
 int grid_for(K kernel, uint64_t items, int* grid) {
   int cap;
   int rc = resident_blocks(kernel, &cap);
   if (rc) return rc;
-  const uint64_t want = (items * T + kBlock - 1) / kBlock;
-  *grid = (int)std::max<uint64_t>(1, std::min<uint64_t>(want, (uint64_t)cap));
+  const uint64_t per_block = kBlock / T;  // work units per block
+  const uint64_t cap_items = (uint64_t)cap * per_block;
+  uint64_t want = items;
+  if (items > cap_items) {
+    want = cap_items;
+    if (balance_rounds()) {
+      const uint64_t rounds = (items + cap_items - 1) / cap_items;
+      want = (items + rounds - 1) / rounds;
+    }
+  }
+  *grid = (int)std::max<uint64_t>(1, (want + per_block - 1) / per_block);
   return FLB_OK;
 }
 

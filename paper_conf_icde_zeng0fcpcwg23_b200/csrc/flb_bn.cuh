@@ -244,7 +244,7 @@ __device__ __forceinline__ uint32_t collapse(uint32_t (&r)[X], const uint32_t (&
 // its word b_i with one LDS that every lane of the group hits at the same address (a broadcast),
 // replacing a register-file copy of b plus a shuffle.  Lane k's chunk sits at k*LD with LD = X+4
 // so the 16-byte stores of the T lanes hit distinct bank quads.  Blocks have <= kMaxWarps warps.
-constexpr int kMaxWarps = 4;
+constexpr int kMaxWarps = 1;  // flb_api.cu launches one-warp blocks
 
 template <int X>
 __device__ __forceinline__ uint32_t* stage_base() {
