@@ -50,6 +50,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-sample-seconds", type=float, default=20.0)
+    ap.add_argument("--workload", choices=["c2", "c1", "c3", "c4", "c5"], default="c2",
+                    help="BASELINE.json configs: c2 (default, the headline) or c1/c3/c4/c5 (single GPU)")
+    ap.add_argument("--c5-ops", type=int, default=0, help="c5 batch per key size (default: 1M / 256K)")
     ap.add_argument("--encrypt", choices=["keyholder", "public"], default="keyholder",
                     help="C2 clients hold the key pair (they decrypt the aggregate, Fig. 2), so they may "
                          "encrypt by CRT; 'public' uses the public-key-only kernel")
@@ -461,10 +464,222 @@ def run_flb(args):
     return 0
 
 
+# ----------------------------------------------------------------------------- other configs
+def _timer():
+    import torch
+    ev = {}
+
+    def mark(name):
+        e = torch.cuda.Event(enable_timing=True)
+        e.record()
+        ev.setdefault(name, []).append(e)
+    return ev, mark
+
+
+def _phases(ev, names, steps):
+    out = {n: 0.0 for n in names[1:]}
+    total = []
+    for s in range(steps):
+        total.append(ev[names[0]][s].elapsed_time(ev[names[-1]][s]))
+        for a, b in zip(names[:-1], names[1:]):
+            out[b] += ev[a][s].elapsed_time(ev[b][s]) / steps
+    return sum(total) / len(total), out
+
+
+def run_other(args):
+    """C1, C3, C4, C5 on one GPU (BASELINE.json configs[0], [2], [3], [4])."""
+    import numpy as np
+    import torch
+    import paper_conf_icde_zeng0fcpcwg23_b200 as flb
+    import synthetic
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    wl = args.workload
+    clk = ClockSampler(0)
+    res = {"metric": METRIC, "unit": UNIT, "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+           "dtype": "u32-limb bigint (+f64 codec)", "data": "synthetic"}
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    clk.start()
+
+    def run_steps(step, names):
+        for s in range(args.warmup):
+            step(s)
+        torch.cuda.synchronize()
+        ev.clear()
+        for s in range(args.steps):
+            flush.zero_()
+            step(100 + s)
+        torch.cuda.synchronize()
+        return _phases(ev, names, args.steps)
+
+    ev, mark = _timer()
+    if wl == "c1":
+        pub, priv = flb.keygen(1024, 0xF1B0 + 1024)
+        cd = flb.Codec(0.5, 30, 2, 1)
+        a, b = synthetic.c1_values()
+        ta, tb = torch.from_numpy(a).to(dev), torch.from_numpy(b).to(dev)
+        nv = len(a)
+        pts = torch.empty((2 * nv, pub.pt_words), dtype=torch.int32, device=dev)
+        cts = torch.empty((3 * nv, pub.ct_words), dtype=torch.int32, device=dev)
+        dec = torch.empty((3 * nv, pub.pt_words), dtype=torch.int32, device=dev)
+        out = torch.empty(3 * nv, dtype=torch.float32, device=dev)
+
+        def step(s):
+            mark("t0")
+            flb.pack(pub, cd, ta, out=pts[:nv])
+            flb.pack(pub, cd, tb, out=pts[nv:])
+            mark("pack")
+            flb.encrypt(pub, pts, seed=s, out=cts[:2 * nv])
+            mark("encrypt")
+            flb.add(pub, cts[:nv], cts[nv:2 * nv], out=cts[2 * nv:])
+            mark("add")
+            flb.decrypt(priv, cts, out=dec)
+            mark("decrypt")
+            flb.unpack(pub, cd, dec[:2 * nv], 2 * nv, summands=1, out=out[:2 * nv])
+            flb.unpack(pub, cd, dec[2 * nv:], nv, summands=2, out=out[2 * nv:])
+            mark("unpack")
+        names = ["t0", "pack", "encrypt", "add", "decrypt", "unpack"]
+        ms, ph = run_steps(step, names)
+        ops = 2 * nv + nv + 3 * nv
+        res.update(value=ops / (ms * 1e-3), ms_per_step=ms, breakdown_ms=ph,
+                   ops_per_step={"encrypt": 2 * nv, "add": nv, "decrypt": 3 * nv},
+                   config={"workload": "C1: 1024-bit key, 1,000 fixed-point values a, b ~ U(-0.5, 0.5); "
+                                       "encrypt 2,000, pairwise hom-add 1,000, decrypt 3,000 (latency point: "
+                                       "cannot fill 148 SMs)", "key_bits": 1024, "codec": "alpha=0.5 rho=30 b=2 S=1"})
+    elif wl == "c3":
+        pub, priv = flb.keygen(2048, 0xF1B0 + 2048)
+        N, F = 1 << 22, 8
+        d, x = synthetic.c3_residuals(N, F)
+        cd = flb.Codec(1.0, 30, 2, 1)
+        td = torch.from_numpy(d).to(dev)
+        tx = torch.from_numpy(x.view(np.int32).reshape(N * F, 1)).to(dev)
+        pt = torch.empty((N, pub.pt_words), dtype=torch.int32, device=dev)
+        ct = torch.empty((N, pub.ct_words), dtype=torch.int32, device=dev)
+        ctf = torch.empty((N * F, pub.ct_words), dtype=torch.int32, device=dev)
+        i = torch.arange(N, dtype=torch.int64, device=dev)
+        idx = torch.cat([i * F + f for f in range(F)])
+        offs = torch.arange(F + 1, dtype=torch.int64, device=dev) * N
+        agg = torch.empty((F, pub.ct_words), dtype=torch.int32, device=dev)
+        rep = torch.arange(N * F, dtype=torch.int64, device=dev) // F
+
+        def step(s):
+            mark("t0")
+            flb.pack(pub, cd, td, out=pt)
+            mark("pack")
+            if args.encrypt == "keyholder":
+                flb.encrypt_crt(priv, pt, seed=s, out=ct)
+            else:
+                flb.encrypt(pub, pt, seed=s, out=ct)
+            mark("encrypt")
+            flb.scalar_mul(pub, ct.index_select(0, rep), tx, out=ctf)
+            mark("scalar_mul")
+            flb.reduce_segments(pub, ctf, offs, idx=idx, max_segment_len=N, out=agg)
+            mark("reduce")
+            flb.decrypt(priv, agg)
+            mark("decrypt")
+        names = ["t0", "pack", "encrypt", "scalar_mul", "reduce", "decrypt"]
+        ms, ph = run_steps(step, names)
+        ops = N + N * F + N * F + F
+        res.update(value=ops / (ms * 1e-3), ms_per_step=ms, breakdown_ms=ph,
+                   ops_per_step={"encrypt": N, "scalar_mul": N * F, "add": N * F, "decrypt": F},
+                   config={"workload": "C3 Hetero LR: 2048-bit key, 4,194,304 encrypted residuals (%s), "
+                                       "x 8 u32 feature scalars each (scalar-mul), product per feature, "
+                                       "decrypt 8" % args.encrypt, "key_bits": 2048,
+                           "note": "the ciphertext replication for the 8 features (index_select) is inside "
+                                   "the scalar_mul phase"})
+    elif wl == "c4":
+        pub, priv = flb.keygen(2048, 0xF1B0 + 2048)
+        nsamp, bins = 1 << 20, 256
+        gh, bb, offsets, idx = synthetic.c4_histogram(n=nsamp, bins=bins)
+        cd = flb.Codec(1.0, 44, 20, 2)
+        tgh = torch.from_numpy(gh).to(dev)
+        toff, tidx = torch.from_numpy(offsets).to(dev), torch.from_numpy(idx).to(dev)
+        cnt = torch.from_numpy(np.diff(offsets).astype(np.int32)).to(dev)
+        maxlen = int(np.diff(offsets).max())
+        pt = torch.empty((nsamp, pub.pt_words), dtype=torch.int32, device=dev)
+        ct = torch.empty((nsamp, pub.ct_words), dtype=torch.int32, device=dev)
+        agg = torch.empty((bins, pub.ct_words), dtype=torch.int32, device=dev)
+
+        def step(s):
+            mark("t0")
+            flb.pack(pub, cd, tgh, out=pt)
+            mark("pack")
+            if args.encrypt == "keyholder":
+                flb.encrypt_crt(priv, pt, seed=s, out=ct)
+            else:
+                flb.encrypt(pub, pt, seed=s, out=ct)
+            mark("encrypt")
+            flb.reduce_segments(pub, ct, toff, idx=tidx, max_segment_len=maxlen, out=agg)
+            mark("reduce")
+            dd = flb.decrypt(priv, agg)
+            mark("decrypt")
+            flb.unpack(pub, cd, dd, 2 * bins, summands=cnt)
+            mark("unpack")
+        names = ["t0", "pack", "encrypt", "reduce", "decrypt", "unpack"]
+        ms, ph = run_steps(step, names)
+        ops = nsamp + (nsamp - bins) + bins
+        res.update(value=ops / (ms * 1e-3), ms_per_step=ms, breakdown_ms=ph,
+                   ops_per_step={"encrypt": nsamp, "add": nsamp - bins, "decrypt": bins},
+                   config={"workload": "C4 Hetero SBT: 2048-bit key, 1,048,576 samples, (g, h) in two 64-bit "
+                                       "slots (rho=44, b=20), encrypt (%s), segmented product into 256 "
+                                       "quantile bins, decrypt 256, unpack with bin counts" % args.encrypt,
+                           "key_bits": 2048})
+    elif wl == "c5":
+        per = {}
+        for bits in (1024, 2048, 3072, 4096):
+            M = args.c5_ops or ((1 << 20) if bits <= 2048 else (1 << 18))
+            pub, priv = flb.keygen(bits, 0xF1B0 + bits)
+            p, q, n = priv.export()
+            base = synthetic.ints_to_limbs(synthetic.uniform_below(n, 256, 5 + bits), pub.pt_words).view(np.int32)
+            m = torch.from_numpy(base).to(dev).repeat(M // 256, 1)
+            c = torch.empty((M, pub.ct_words), dtype=torch.int32, device=dev)
+            o = torch.empty_like(c)
+            dm = torch.empty_like(m)
+            ev.clear()
+
+            def step(s):
+                mark("t0")
+                flb.encrypt(pub, m, seed=s, out=c)
+                mark("enc")
+                flb.encrypt_crt(priv, m, seed=s, out=o)
+                mark("enc_crt")
+                flb.decrypt(priv, c, out=dm)
+                mark("dec")
+                flb.add(pub, c, o, out=o)
+                mark("add")
+            names = ["t0", "enc", "enc_crt", "dec", "add"]
+            ms, ph = run_steps(step, names)
+            lp = {k: flb.op_cost(priv if k in ("decrypt", "encrypt_crt") else pub, k)[1]
+                  for k in ("encrypt", "encrypt_crt", "decrypt", "add")}
+            peak = 148 * PEAK_LP_PER_CLK_SM * 1965e6
+            per[str(bits)] = {
+                "batch": M,
+                "encrypt_per_s": M / (ph["enc"] * 1e-3), "encrypt_keyholder_per_s": M / (ph["enc_crt"] * 1e-3),
+                "decrypt_per_s": M / (ph["dec"] * 1e-3), "add_per_s": M / (ph["add"] * 1e-3),
+                "frac_roofline": {"encrypt": lp["encrypt"] * M / (ph["enc"] * 1e-3) / peak,
+                                  "encrypt_keyholder": lp["encrypt_crt"] * M / (ph["enc_crt"] * 1e-3) / peak,
+                                  "decrypt": lp["decrypt"] * M / (ph["dec"] * 1e-3) / peak,
+                                  "add": lp["add"] * M / (ph["add"] * 1e-3) / peak}}
+            del c, o, dm, m
+        v = per["2048"]
+        res.update(value=3.0 / (1 / v["encrypt_per_s"] + 1 / v["decrypt_per_s"] + 1 / v["add_per_s"]),
+                   ms_per_step=None, per_key=per,
+                   config={"workload": "C5 key sweep 1024/2048/3072/4096: encrypt (public and key-holder), "
+                                       "decrypt, add on uniform m < n; batch 1,048,576 (1024/2048) and 262,144 "
+                                       "(3072/4096) per op instead of 16M (time budget)",
+                           "value_definition": "2048-bit enc/dec/add mix: 3 / sum of per-op seconds"})
+    res["clocks"] = clk.stop()
+    print(json.dumps(res), flush=True)
+    return 0
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
+    if args.workload != "c2":
+        return run_other(args)
     return run_flb(args)
 
 
