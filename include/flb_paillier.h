@@ -147,6 +147,34 @@ int flb_unpack(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt, s
 int flb_unpack_sums(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt,
                     size_t n_values, uint64_t* sums, void* stream);
 
+/* ---------------------------------------------------------------- host-buffer pipeline (NEXT-1)
+ * PAPER Fig. 4 / §V-A (L288–L298): host data -> compression -> copy to GPU -> HE -> copy back.
+ * These take HOST pointers (pageable or pinned), split the batch into 32,768-element chunks and
+ * overlap each chunk's H2D copy, kernels and D2H copy with the host-side copy of the previous
+ * chunk on two internal streams of the current device.  They block until the host output is
+ * complete.  Scratch (pinned staging, device buffers) is per device and reused across calls;
+ * calls on one device are serialised.  Results are bit-identical to the device-buffer calls. */
+
+/* ①–④: x_host float32 [n_values] -> quantise + pack (codec) -> encrypt (key-holder CRT path when
+ * priv is non-NULL, else the public path; r from Philox(seed, ctr0 + plaintext index)) ->
+ * c_host [ceil(n_values/slots)][ct_words].  Errors: FLB_EINVAL, FLB_ECUDA, as the batch calls. */
+int flb_pack_encrypt_host(const flb_pub* pub, const flb_priv* priv, const flb_codec* codec,
+                          const float* x_host, size_t n_values, uint64_t seed, uint64_t ctr0,
+                          uint32_t* c_host);
+
+/* ⑤–⑨: c_host [ceil(n_values/slots)][ct_words] -> decrypt -> unpack + dequantise -> x_host
+ * float32 [n_values]; summands_host: uint32 [ceil(n_values/slots)] or NULL (then
+ * summands_scalar).  pub must be priv's public key.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_decrypt_unpack_host(const flb_priv* priv, const flb_pub* pub, const flb_codec* codec,
+                            const uint32_t* c_host, size_t n_values, const uint32_t* summands_host,
+                            uint32_t summands_scalar, float* x_host);
+
+/* ④⑤ homomorphic aggregation: flb_reduce_segments over host buffers (c_host
+ * [num_inputs][ct_words], idx_host/offsets_host int64, out_host [num_segments][ct_words]). */
+int flb_reduce_segments_host(const flb_pub* pub, const uint32_t* c_host, size_t num_inputs,
+                             const int64_t* idx_host, const int64_t* offsets_host,
+                             size_t num_segments, size_t max_segment_len, uint32_t* out_host);
+
 /* Debug entry for the Montgomery primitive (PAPER Alg. 2): out_i = a_i b_i R^-1
  * mod n^2, R = 2^(32 ct_words), canonical.  a_i < n^2, b_i < n^2.  [count][ct_words]. */
 int flb_debug_mont_mul(const flb_pub* pub, const uint32_t* a, const uint32_t* b, uint32_t* out,

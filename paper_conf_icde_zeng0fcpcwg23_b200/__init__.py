@@ -22,7 +22,8 @@ from ._lib import LIB, FlbError, check
 __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
-    "Codec", "FlbError", "library_path", "op_cost",
+    "Codec", "FlbError", "library_path", "op_cost", "pack_encrypt_host", "decrypt_unpack_host",
+    "reduce_segments_host",
 ]
 
 library_path = _lib.LIB_PATH
@@ -263,6 +264,65 @@ def unpack_sums(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int, o
     cs = codec.struct()
     check("flb_unpack_sums", LIB.flb_unpack_sums(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, _ptr(out),
                                                  _stream(stream)))
+    return out
+
+
+# ----------------------------------------------------------------------------- host-buffer pipeline
+def _np_ptr(a):
+    import numpy as np
+    if not isinstance(a, np.ndarray) or not a.flags["C_CONTIGUOUS"]:
+        raise ValueError("host buffers must be C-contiguous numpy arrays")
+    return a.ctypes.data
+
+
+def pack_encrypt_host(pub: PublicKey, codec: Codec, x, seed: int = 0, ctr0: int = 0,
+                      priv: Optional[PrivateKey] = None, out=None):
+    """Host float32 values -> host ciphertext limbs [M, ct_words] (uint32), pipelined (PAPER Fig. 4 ①–④).
+    With ``priv`` the key-holder CRT encryption is used (same bits)."""
+    import numpy as np
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    M = codec.num_plaintexts(x.shape[0])
+    if out is None:
+        out = np.empty((M, pub.ct_words), dtype=np.uint32)
+    cs = codec.struct()
+    check("flb_pack_encrypt_host", LIB.flb_pack_encrypt_host(pub.handle, priv.handle if priv else None,
+                                                             ctypes.byref(cs), _np_ptr(x), x.shape[0],
+                                                             seed & 0xFFFFFFFFFFFFFFFF, ctr0, _np_ptr(out)))
+    return out
+
+
+def decrypt_unpack_host(priv: PrivateKey, codec: Codec, c, n_values: int, summands=1, out=None):
+    """Host ciphertexts -> host float32 values, pipelined (PAPER Fig. 4 ⑤–⑨)."""
+    import numpy as np
+    c = np.ascontiguousarray(c, dtype=np.uint32)
+    if out is None:
+        out = np.empty((n_values,), dtype=np.float32)
+    cs = codec.struct()
+    if isinstance(summands, int):
+        sp, ss = None, summands
+    else:
+        summands = np.ascontiguousarray(summands, dtype=np.uint32)
+        sp, ss = _np_ptr(summands), 0
+    check("flb_decrypt_unpack_host", LIB.flb_decrypt_unpack_host(priv.handle, priv.pub.handle, ctypes.byref(cs),
+                                                                 _np_ptr(c), n_values, sp, ss, _np_ptr(out)))
+    return out
+
+
+def reduce_segments_host(pub: PublicKey, c, offsets, idx=None, max_segment_len: int = 0, out=None):
+    """Segmented ciphertext product over host buffers."""
+    import numpy as np
+    c = np.ascontiguousarray(c, dtype=np.uint32)
+    offsets = np.ascontiguousarray(offsets, dtype=np.int64)
+    S = offsets.shape[0] - 1
+    ip = None
+    if idx is not None:
+        idx = np.ascontiguousarray(idx, dtype=np.int64)
+        ip = _np_ptr(idx)
+    if out is None:
+        out = np.empty((S, pub.ct_words), dtype=np.uint32)
+    check("flb_reduce_segments_host", LIB.flb_reduce_segments_host(pub.handle, _np_ptr(c), c.shape[0], ip,
+                                                                   _np_ptr(offsets), S, max_segment_len,
+                                                                   _np_ptr(out)))
     return out
 
 

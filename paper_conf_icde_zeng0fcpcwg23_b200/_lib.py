@@ -54,6 +54,9 @@ SIGNATURES = {
     "flb_unpack": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P, _P]),
     "flb_unpack_sums": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _P]),
     "flb_debug_mont_mul": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
+    "flb_pack_encrypt_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _U64, _U64, _P]),
+    "flb_decrypt_unpack_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P]),
+    "flb_reduce_segments_host": (ctypes.c_int, [_P, _P, _SZ, _P, _P, _SZ, _SZ, _P]),
     "flb_op_cost": (ctypes.c_int, [_P, _P, ctypes.c_int, ctypes.POINTER(_U64), ctypes.POINTER(_U64)]),
     "flb_last_error": (ctypes.c_char_p, []),
     "flb_version": (ctypes.c_char_p, []),

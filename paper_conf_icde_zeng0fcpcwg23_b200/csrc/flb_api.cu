@@ -96,6 +96,10 @@ int frame_for_bits(size_t nbits) {
 
 }  // namespace
 
+namespace flb {
+void set_last_error(const std::string& msg) { g_err = msg; }
+}  // namespace flb
+
 // ----------------------------------------------------------------------------- key structs
 struct flb_pub {
   uint32_t nbits = 0, frame = 0, s = 0, sp = 0;

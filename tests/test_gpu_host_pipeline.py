@@ -1,0 +1,60 @@
+"""The host-buffer pipeline (flb_*_host, NEXT-1 / PAPER Fig. 4) gives the same bits as the
+device-buffer calls, across several chunks with a ragged tail; sampled outputs vs the oracle."""
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_icde_zeng0fcpcwg23_b200 as flb  # noqa: E402
+import synthetic  # noqa: E402
+from oracle import codec, paillier, philox  # noqa: E402
+from paper_conf_icde_zeng0fcpcwg23_b200 import dist as fdist  # noqa: E402
+from tests.helpers import golden_keys  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("keyholder", [True, False])
+def test_c2_round_through_host_buffers(keyholder):
+    p, q = golden_keys()["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    S, clients = 31, 3
+    cd = flb.Codec(1.0, 29, 3, S)
+    nv = 70000 * S + 17          # 70,001 plaintexts per client: 3 chunks of 32,768, ragged tail
+    xs = [synthetic.c2_gradient(c, n=nv) for c in range(clients)]
+    rows = cd.num_plaintexts(nv)
+    cts = np.concatenate([flb.pack_encrypt_host(pub, cd, xs[c], seed=9, ctr0=c * rows,
+                                                priv=priv if keyholder else None) for c in range(clients)])
+    # same bits as the device path
+    dev = torch.cat([flb.pack(pub, cd, torch.from_numpy(x).cuda()) for x in xs])
+    ref = flb.encrypt(pub, dev, seed=9).cpu().numpy().view(np.uint32)
+    assert np.array_equal(cts, ref)
+    i = clients * rows - 1
+    z = codec.pack([float(v) for v in xs[-1][(rows - 1) * S:]], 1.0, 29, 3, S)[0]
+    assert synthetic.limbs_to_ints(cts[i:i + 1])[0] == paillier.encrypt(n, z, philox.draw_r(n, 9, i, pub.pt_words))
+    offs, idx = fdist.client_segments(clients, rows)
+    agg = flb.reduce_segments_host(pub, cts, offs.numpy(), idx.numpy(), max_segment_len=clients)
+    agg_dev = flb.reduce_segments(pub, torch.from_numpy(cts.view(np.int32)).cuda(), offs.cuda(),
+                                  idx=idx.cuda(), max_segment_len=clients).cpu().numpy().view(np.uint32)
+    assert np.array_equal(agg, agg_dev)
+    out = flb.decrypt_unpack_host(priv, cd, agg, nv, summands=clients)
+    dec = flb.decrypt(priv, torch.from_numpy(agg.view(np.int32)).cuda())
+    out_dev = flb.unpack(pub, cd, dec, nv, summands=clients).cpu().numpy()
+    assert np.array_equal(out.view(np.uint32), out_dev.view(np.uint32))
+    exact = np.sum(np.array(xs, dtype=np.float64), axis=0)
+    assert np.max(np.abs(out - exact)) <= clients / ((1 << 29) - 1) + 1e-6
+
+
+def test_decrypt_unpack_host_per_plaintext_counts():
+    p, q = golden_keys()["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    cd = flb.Codec(1.0, 44, 20, 2)
+    x = np.random.default_rng(3).uniform(-1, 1, 2 * 40000).astype(np.float32)
+    c = flb.pack_encrypt_host(pub, cd, x, seed=4)
+    cnt = np.ones(c.shape[0], dtype=np.uint32)
+    out = flb.decrypt_unpack_host(priv, cd, c, x.shape[0], summands=cnt)
+    assert np.max(np.abs(out - x)) <= 1.0 / ((1 << 44) - 1) + np.abs(x).max() * 2 ** -24
