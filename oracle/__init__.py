@@ -35,4 +35,4 @@ Parity status per function (DESIGN.md §3 lists the pins):
 * montgomery.mont_mul — pinned (definition a*b*R^-1 mod N checked by multiplying back).
 """
 
-from . import paillier, philox, codec, montgomery  # noqa: F401
+from . import paillier, philox, codec, montgomery, modarith  # noqa: F401
