@@ -38,6 +38,7 @@ extern "C" {
 
 typedef struct flb_pub flb_pub;   /* n, n^2, Montgomery constants, encryption schedule */
 typedef struct flb_priv flb_priv; /* p, q, p^2, q^2, CRT constants, decryption schedules */
+typedef struct flb_mod flb_mod;   /* any odd modulus (Table I mod_mul / mod_pow, RSA)             */
 
 enum {
   FLB_OK = 0,
@@ -146,6 +147,40 @@ int flb_unpack(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt, s
 /* The exact slot integers Sum_i (device uint64 [n_values]).  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_unpack_sums(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt,
                     size_t n_values, uint64_t* sums, void* stream);
+
+/* ---------------------------------------------------------------- generic modular API, RSA (NEXT-4)
+ * PAPER Table I (L236–L256) and §IV-D (L269–L284): mod_mul(values1, values2, n) and
+ * mod_pow(x, p, n) over batches, with the same thread-group Montgomery kernels; RSA (L247–L251)
+ * is key_gen below + mod_pow_shared (encrypt m^e, decrypt c^d) + mod_mul (the multiplicative
+ * homomorphism).  A modulus of W limbs uses the smallest frame of 32/64/96/128/192/256 limbs >= W;
+ * batch operands are [count][flb_mod_words] limbs, each < n. */
+
+/* Create a modulus handle from host limbs (odd n >= 3, at most 8192 bits).  Errors: FLB_EINVAL,
+ * FLB_EUNSUPPORTED (> 8192 bits). */
+int flb_mod_create(const uint32_t* n, uint32_t words, flb_mod** out);
+void flb_mod_free(flb_mod* mod);
+uint32_t flb_mod_words(const flb_mod* mod); /* frame limbs of a batch element */
+
+/* out_i = a_i b_i mod n (Table I mod_mul, L245; RSA::mul, L250). */
+int flb_mod_mul(const flb_mod* mod, const uint32_t* a, const uint32_t* b, uint32_t* out,
+                size_t count, void* stream);
+
+/* out_i = base_i ^ e_i mod n with per-element exponents e [count][e_words] on the device
+ * (Table I mod_pow, L246); e_i = 0 gives 1. */
+int flb_mod_pow(const flb_mod* mod, const uint32_t* base, const uint32_t* e, uint32_t e_words,
+                uint32_t* out, size_t count, void* stream);
+
+/* out_i = base_i ^ e mod n with one exponent for the batch, given in HOST memory (its sliding-
+ * window schedule is built once per exponent and cached on the handle): RSA::encrypt (e) and
+ * RSA::decrypt (d), L248–L249. */
+int flb_mod_pow_shared(const flb_mod* mod, const uint32_t* base, const uint32_t* e_host,
+                       uint32_t e_words, uint32_t* out, size_t count, void* stream);
+
+/* RSA::key_gen (L247, L281), host, deterministic in seed: p > q primes of key_bits/2 bits
+ * (Miller–Rabin), n = p q with bits(n) = key_bits, d = e^-1 mod (p-1)(q-1).  n_out, d_out:
+ * key_bits/32 limbs; p_out, q_out: key_bits/64 limbs (any may be NULL). */
+int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out, uint32_t* d_out,
+                   uint32_t* p_out, uint32_t* q_out);
 
 /* ---------------------------------------------------------------- host-buffer pipeline (NEXT-1)
  * PAPER Fig. 4 / §V-A (L288–L298): host data -> compression -> copy to GPU -> HE -> copy back.

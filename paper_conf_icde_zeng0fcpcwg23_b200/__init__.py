@@ -22,7 +22,7 @@ from ._lib import LIB, FlbError, check
 __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
-    "Codec", "FlbError", "library_path", "op_cost", "pack_encrypt_host", "decrypt_unpack_host",
+    "Codec", "FlbError", "library_path", "op_cost", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
     "reduce_segments_host",
 ]
 
@@ -265,6 +265,58 @@ def unpack_sums(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int, o
     check("flb_unpack_sums", LIB.flb_unpack_sums(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, _ptr(out),
                                                  _stream(stream)))
     return out
+
+
+# ----------------------------------------------------------------------------- Table I generic API, RSA
+class Modulus:
+    """An odd modulus for Table I's mod_mul / mod_pow and RSA (L247–L251)."""
+
+    def __init__(self, n: int):
+        words = max(1, (n.bit_length() + 31) // 32)
+        h = ctypes.c_void_p()
+        check("flb_mod_create", LIB.flb_mod_create(_limbs_of(n, words), words, ctypes.byref(h)))
+        self._h, self.n = h, n
+        self.words = LIB.flb_mod_words(h)
+
+    def __del__(self, _free=LIB.flb_mod_free):
+        h, self._h = getattr(self, "_h", None), None
+        if h:
+            _free(h)
+
+    def mul(self, a: torch.Tensor, b: torch.Tensor, out=None, stream=None) -> torch.Tensor:
+        M = _check_batch(a, self.words, "a")
+        _check_batch(b, self.words, "b")
+        out = torch.empty_like(a) if out is None else out
+        check("flb_mod_mul", LIB.flb_mod_mul(self._h, _ptr(a), _ptr(b), _ptr(out), M, _stream(stream)))
+        return out
+
+    def pow(self, base: torch.Tensor, e: torch.Tensor, out=None, stream=None) -> torch.Tensor:
+        """Per-element exponents e [count, e_words] (device)."""
+        M = _check_batch(base, self.words, "base")
+        _check_batch(e, e.shape[1], "e")
+        out = torch.empty_like(base) if out is None else out
+        check("flb_mod_pow", LIB.flb_mod_pow(self._h, _ptr(base), _ptr(e), e.shape[1], _ptr(out), M,
+                                             _stream(stream)))
+        return out
+
+    def pow_shared(self, base: torch.Tensor, e: int, out=None, stream=None) -> torch.Tensor:
+        """One exponent (a Python int) for the whole batch."""
+        M = _check_batch(base, self.words, "base")
+        ew = max(1, (e.bit_length() + 31) // 32)
+        out = torch.empty_like(base) if out is None else out
+        check("flb_mod_pow_shared", LIB.flb_mod_pow_shared(self._h, _ptr(base), _limbs_of(e, ew), ew, _ptr(out), M,
+                                                           _stream(stream)))
+        return out
+
+
+def rsa_keygen(key_bits: int, seed: int, e: int = 65537) -> Tuple[int, int, int, int, int]:
+    """RSA::key_gen (PAPER L247): (n, e, d, p, q) as Python ints (host C++ keygen)."""
+    w = key_bits // 32
+    n, d = (ctypes.c_uint32 * w)(), (ctypes.c_uint32 * w)()
+    p, q = (ctypes.c_uint32 * (w // 2))(), (ctypes.c_uint32 * (w // 2))()
+    check("flb_rsa_keygen", LIB.flb_rsa_keygen(key_bits, seed & 0xFFFFFFFFFFFFFFFF, e, n, d, p, q))
+    to_int = lambda a: sum(int(x) << (32 * i) for i, x in enumerate(a))
+    return to_int(n), e, to_int(d), to_int(p), to_int(q)
 
 
 # ----------------------------------------------------------------------------- host-buffer pipeline

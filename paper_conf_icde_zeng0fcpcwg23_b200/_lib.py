@@ -54,6 +54,13 @@ SIGNATURES = {
     "flb_unpack": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P, _P]),
     "flb_unpack_sums": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _P]),
     "flb_debug_mont_mul": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
+    "flb_mod_create": (ctypes.c_int, [_P, _U32, ctypes.POINTER(_P)]),
+    "flb_mod_free": (None, [_P]),
+    "flb_mod_words": (_U32, [_P]),
+    "flb_mod_mul": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
+    "flb_mod_pow": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),
+    "flb_mod_pow_shared": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),
+    "flb_rsa_keygen": (ctypes.c_int, [_U32, _U64, _U32, _P, _P, _P, _P]),
     "flb_pack_encrypt_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _U64, _U64, _P]),
     "flb_decrypt_unpack_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P]),
     "flb_reduce_segments_host": (ctypes.c_int, [_P, _P, _SZ, _P, _P, _SZ, _SZ, _P]),

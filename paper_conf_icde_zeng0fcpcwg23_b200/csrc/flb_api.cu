@@ -129,6 +129,29 @@ struct flb_priv {
   ~flb_priv() { delete pub; }
 };
 
+// A generic odd modulus for Table I's mod_mul / mod_pow and RSA (L247–L251): the
+// Montgomery constants live in an flb_pub "core" whose n2 slot holds the modulus, so the hom-add and
+// scalar-mul kernels serve mod_mul and per-element mod_pow unchanged.
+struct flb_mod {
+  flb_pub core;
+  std::mutex mu;
+  struct Sched {
+    H::Schedule s;
+    std::map<int, uint32_t*> dev;
+  };
+  std::map<std::vector<uint32_t>, Sched> scheds;  // batch-shared exponents seen so far
+  ~flb_mod() {
+    int cur;
+    if (cudaGetDevice(&cur) != cudaSuccess) return;
+    for (auto& kv : scheds)
+      for (auto& d : kv.second.dev) {
+        cudaSetDevice(d.first);
+        cudaFree(d.second);
+      }
+    cudaSetDevice(cur);
+  }
+};
+
 namespace {
 
 flb_pub* make_pub(const Limbs& n_in) {
@@ -215,6 +238,22 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
   V->o_qR_n = V->blob.put(Cn.to(V->q), sp);
   V->o_qinvR_p = V->blob.put(Cp.to(H::inv_mod_prime(V->q, V->p)), sp);
   return V;
+}
+
+flb_mod* make_mod(const Limbs& n_in, uint32_t S) {
+  auto* M = new flb_mod();
+  flb_pub& K = M->core;
+  K.nbits = (uint32_t)H::bits(n_in);
+  K.s = S;
+  K.sp = S / 2;
+  K.frame = 16 * S;  // the dispatch key: S limbs is the "n^2" frame of a 16*S... i.e. 1024 <-> 64 limbs
+  K.n2 = H::resized(n_in, S);
+  H::MontCtx C(K.n2);
+  K.n2_n0inv = C.n0inv;
+  K.o_n2 = K.blob.put(K.n2, S);
+  K.o_R2 = K.blob.put(C.R2, S);
+  K.o_R1 = K.blob.put(C.R1, S);
+  return M;
 }
 
 // ----------------------------------------------------------------------------- launching
@@ -406,6 +445,31 @@ int run_encrypt_crt(const flb_priv* V, const uint32_t* dev, const uint32_t* m, c
   return FLB_OK;
 }
 
+template <int X, int T>
+int run_modpow(const flb_pub* K, const uint32_t* dev, const uint32_t* sched, const H::Schedule* S, const uint32_t* base,
+               uint32_t* out, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_modpow<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)S->table * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::PowArgs A;
+  A.N = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.sched = sched;
+  A.sched_len = (int)S->ops.size();
+  A.table = S->table;
+  A.base = base;
+  A.out = out;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_modpow<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
 template <int X, int T, bool DEBUG>
 int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
             cudaStream_t st) {
@@ -540,7 +604,9 @@ static int limbs_per_lane() {
   do {                                                                            \
     const bool nar = limbs_per_lane() == 8;                                       \
     switch (frame) {                                                              \
+      case 512: return FN<16, 2>(__VA_ARGS__);  /* generic moduli of <= 32 limbs */ \
       case 1024: return nar ? FN<8, 8>(__VA_ARGS__) : FN<16, 4>(__VA_ARGS__);     \
+      case 1536: return FN<12, 8>(__VA_ARGS__); /* generic moduli of <= 96 limbs */ \
       case 2048: return nar ? FN<8, 16>(__VA_ARGS__) : FN<16, 8>(__VA_ARGS__);    \
       case 3072: return FN<12, 16>(__VA_ARGS__);                                  \
       case 4096: return nar ? FN<8, 32>(__VA_ARGS__) : FN<16, 16>(__VA_ARGS__);   \
@@ -765,6 +831,128 @@ int flb_reduce_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs, 
   if (rc) return rc;
   FLB_DISPATCH_ENC(K->frame, run_reduce, K, dev, c, num_inputs, idx, offsets, num_segments, max_segment_len, out,
                    (cudaStream_t)stream);
+}
+
+static int grid_1d(uint64_t n);
+
+int flb_mod_create(const uint32_t* n, uint32_t words, flb_mod** out) {
+  if (!n || !out || words == 0) return fail(FLB_EINVAL, "null pointer or zero size");
+  try {
+    Limbs N(n, n + words);
+    const size_t b = H::bits(N);
+    if (b < 2 || !(N[0] & 1)) return fail(FLB_EINVAL, "modulus must be odd and >= 3");
+    uint32_t S = 0;
+    for (uint32_t f : {32u, 64u, 96u, 128u, 192u, 256u})
+      if (b <= 32u * f) { S = f; break; }
+    if (!S) return fail(FLB_EUNSUPPORTED, "modulus above 8192 bits");
+    *out = make_mod(N, S);
+    return FLB_OK;
+  } catch (const std::bad_alloc&) {
+    return fail(FLB_ENOMEM, "host allocation failed");
+  } catch (const std::exception& ex) {
+    return fail(FLB_EINVAL, ex.what());
+  }
+}
+
+void flb_mod_free(flb_mod* M) { delete M; }
+uint32_t flb_mod_words(const flb_mod* M) { return M ? M->core.s : 0; }
+
+int flb_mod_mul(const flb_mod* M, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count, void* stream) {
+  if (!M) return fail(FLB_EINVAL, "null modulus");
+  return flb_add(&M->core, a, b, out, count, stream);
+}
+
+int flb_mod_pow(const flb_mod* M, const uint32_t* base, const uint32_t* e, uint32_t e_words, uint32_t* out,
+                size_t count, void* stream) {
+  if (!M) return fail(FLB_EINVAL, "null modulus");
+  return flb_scalar_mul(&M->core, base, e, e_words, out, count, stream);
+}
+
+int flb_mod_pow_shared(const flb_mod* Mc, const uint32_t* base, const uint32_t* e_host, uint32_t e_words,
+                       uint32_t* out, size_t count, void* stream) {
+  if (!Mc || !base || !e_host || !out || e_words == 0) return fail(FLB_EINVAL, "null pointer or zero size");
+  if (count == 0) return FLB_OK;
+  flb_mod* M = const_cast<flb_mod*>(Mc);
+  const flb_pub* K = &M->core;
+  std::vector<uint32_t> e(e_host, e_host + e_words);
+  while (e.size() > 1 && e.back() == 0) e.pop_back();
+  if (e.size() == 1 && e[0] == 0) {  // x^0 = 1
+    flb::k_fill_one<<<grid_1d(count * K->s), 256, 0, (cudaStream_t)stream>>>(out, count, K->s);
+    FLB_LAUNCH_CHECK();
+    return FLB_OK;
+  }
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  const H::Schedule* S;
+  const uint32_t* sched_dev;
+  {
+    std::lock_guard<std::mutex> lk(M->mu);
+    auto it = M->scheds.find(e);
+    if (it == M->scheds.end()) {
+      try {
+        it = M->scheds.emplace(e, flb_mod::Sched{H::best_schedule(Limbs(e.begin(), e.end()), 7), {}}).first;
+      } catch (const std::exception& ex) {
+        return fail(FLB_EINVAL, ex.what());
+      }
+    }
+    int d;
+    FLB_CK(cudaGetDevice(&d));
+    auto& dv = it->second.dev;
+    if (!dv.count(d)) {
+      uint32_t* p = nullptr;
+      const auto& ops = it->second.s.ops;
+      FLB_CK(cudaMalloc(&p, ops.size() * 4));
+      FLB_CK(cudaMemcpy(p, ops.data(), ops.size() * 4, cudaMemcpyHostToDevice));
+      dv[d] = p;
+    }
+    S = &it->second.s;
+    sched_dev = dv[d];
+  }
+  FLB_DISPATCH_ENC(K->frame, run_modpow, K, dev, sched_dev, S, base, out, count, (cudaStream_t)stream);
+}
+
+int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out, uint32_t* d_out, uint32_t* p_out,
+                   uint32_t* q_out) {
+  if (key_bits < 64 || key_bits > 8192 || key_bits % 64 || e < 3 || !(e & 1))
+    return fail(FLB_EINVAL, "key_bits must be a multiple of 64 in [64, 8192]; e odd >= 3");
+  try {
+    H::Xoshiro256 rng(seed ^ 0x5253412d6b657973ull);
+    const uint32_t w = key_bits / 32;
+    for (;;) {
+      Limbs p = H::random_prime(key_bits / 2, rng), q = H::random_prime(key_bits / 2, rng);
+      if (H::cmp(p, q) == 0) continue;
+      if (H::cmp(p, q) < 0) std::swap(p, q);
+      Limbs n = H::resized(H::mul(p, q), w);
+      if (H::bits(n) != key_bits) continue;
+      Limbs one(p.size(), 0);
+      one[0] = 1;
+      Limbs pm1 = p, qm1 = q;
+      H::sub_in(pm1, one);
+      H::sub_in(qm1, one);
+      const Limbs phi = H::mul(pm1, qm1);
+      const uint32_t r = H::mod_small(phi, e);
+      if (r == 0) continue;  // gcd(e, phi) != 1 (e prime or not: require phi mod e != 0 and check below)
+      // k = -phi^-1 mod e (small), d = (1 + k phi) / e
+      uint64_t inv = 0;
+      for (uint64_t t = 1; t < e; t++)
+        if ((r * t) % e == 1) { inv = t; break; }
+      if (!inv) continue;  // e not coprime to phi
+      const uint32_t k = (uint32_t)((e - inv) % e);
+      Limbs dnum = H::mul_small(phi, k, 1);
+      if (H::mod_small(dnum, e) != 0) continue;
+      Limbs d = H::resized(H::div_small(dnum, e), w + 1);
+      d = H::resized(d, w);
+      if (n_out) for (uint32_t i = 0; i < w; i++) n_out[i] = n[i];
+      if (d_out) for (uint32_t i = 0; i < w; i++) d_out[i] = d[i];
+      Limbs ph = H::resized(p, w / 2), qh = H::resized(q, w / 2);
+      if (p_out) for (uint32_t i = 0; i < w / 2; i++) p_out[i] = ph[i];
+      if (q_out) for (uint32_t i = 0; i < w / 2; i++) q_out[i] = qh[i];
+      return FLB_OK;
+    }
+  } catch (const std::exception& ex) {
+    return fail(FLB_EINVAL, ex.what());
+  }
 }
 
 static int codec_args(const flb_pub* K, const flb_codec* cd, flb::CodecArgs* A) {

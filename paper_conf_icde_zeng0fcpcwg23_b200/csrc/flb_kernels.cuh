@@ -341,6 +341,49 @@ __global__ void __launch_bounds__(32, FLB_MINB_DEC) k_encrypt_crt(const EncCrtAr
   }
 }
 
+// ----------------------------------------------------------------------------- generic mod_pow
+struct PowArgs {
+  ModRef N;                // any odd modulus in the S-limb frame
+  const uint32_t* R2;      // R^2 mod N
+  const uint32_t* sched;   // schedule of the batch-shared exponent
+  int sched_len, table;
+  const uint32_t* base;    // [count][S], each < N
+  uint32_t* out;           // [count][S]
+  uint64_t count;
+  uint32_t* scratch;
+};
+
+// out = base^e mod N for one exponent shared by the batch (Table I mod_pow; RSA
+// encrypt/decrypt, L248–L249).
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_ENC) k_modpow(const PowArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N);
+  const uint32_t n0inv = A.N.n0inv;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t x[X], b[X], acc[X];
+    load_elem<X, T>(x, A.base + e * S, S, valid);
+    load_const<X, T>(b, A.R2);
+    mont_mul<X, T>(x, x, b, n, n0inv);
+    modexp_sched<X, T>(acc, x, A.sched, A.sched_len, A.table, tab, stride, n, n0inv);
+    set_one<X, T>(b);
+    mont_mul<X, T>(acc, acc, b, n, n0inv);
+    if (valid) store_limbs<X>(A.out + e * S + g.k * X, acc);
+  }
+}
+
+// out[i] = 1 (the empty product / x^0), [count][S]
+__global__ void k_fill_one(uint32_t* out, uint64_t count, uint32_t S) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count * S; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = (i % S) == 0 ? 1u : 0u;
+}
+
 // ----------------------------------------------------------------------------- hom-add
 struct AddArgs {
   ModRef N2;

@@ -264,6 +264,31 @@ inline uint32_t mod_small(const Limbs& a, uint32_t d) {
   return (uint32_t)r;
 }
 
+// a * m + add (m, add < 2^32), width grows by one word
+inline Limbs mul_small(const Limbs& a, uint32_t m, uint32_t add = 0) {
+  Limbs r(a.size() + 1, 0);
+  uint64_t c = add;
+  for (size_t i = 0; i < a.size(); i++) {
+    c += (uint64_t)a[i] * m;
+    r[i] = (uint32_t)c;
+    c >>= 32;
+  }
+  r[a.size()] = (uint32_t)c;
+  return r;
+}
+
+// a / d (exact or floor), d < 2^32
+inline Limbs div_small(const Limbs& a, uint32_t d) {
+  Limbs q(a.size(), 0);
+  uint64_t r = 0;
+  for (size_t i = a.size(); i-- > 0;) {
+    const uint64_t cur = (r << 32) | a[i];
+    q[i] = (uint32_t)(cur / d);
+    r = cur % d;
+  }
+  return q;
+}
+
 inline const std::vector<uint32_t>& small_primes() {
   static std::vector<uint32_t> ps = [] {
     std::vector<uint32_t> v;

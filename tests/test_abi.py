@@ -144,3 +144,19 @@ def test_op_cost_matches_independent_window_count():
     bd = sum(min(_sliding_mults(P - 1, w) for w in range(1, 8)) for P in (p, q))
     assert mm_d == bd + 2 * 4 + 2
     assert flb.op_cost(pub, "add") == (2, 2 * (2 * 128 * 128 + 128))
+
+
+def test_mod_create_and_rsa_keygen_host_logic():
+    for bits, words in [(61, 32), (1024, 32), (1025, 64), (2048, 64), (3000, 96), (4096, 128), (8192, 256)]:
+        n = (1 << (bits - 1)) | 1
+        assert flb.Modulus(n).words == words
+    for bad in (0, 1, 2, 10, 1 << 8192):
+        with pytest.raises(flb.FlbError):
+            flb.Modulus(bad)
+    n, e, d, p, q = flb.rsa_keygen(512, 7)
+    assert p > q and p * q == n and n.bit_length() == 512 and e == 65537
+    assert (e * d) % ((p - 1) * (q - 1)) == 1
+    assert all(pow(b, x - 1, x) == 1 for x in (p, q) for b in (2, 3, 5))
+    assert flb.rsa_keygen(512, 7) == (n, e, d, p, q)
+    with pytest.raises(flb.FlbError):
+        flb.rsa_keygen(100, 1)
