@@ -182,6 +182,21 @@ int flb_mod_pow_shared(const flb_mod* mod, const uint32_t* base, const uint32_t*
 int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out, uint32_t* d_out,
                    uint32_t* p_out, uint32_t* q_out);
 
+/* ---------------------------------------------------------------- GPU key generation (NEXT-3)
+ * "random number generator for large integers (including Miller-Rabin large prime
+ * number generator)".  flb_miller_rabin runs `rounds` Miller–Rabin rounds on a batch of odd
+ * candidates (device [count][words], words in {32, 64, 96, 128, 192, 256}, each >= 5), each with
+ * its own modulus; verdict[i] = 1 iff candidate i passed every round.  mont_bases: device
+ * [count][rounds][words] bases in Montgomery form (a~ with 1 <= a~ < P stands for the base
+ * a = a~ 2^(-32 words) mod P), or NULL to draw them from Philox(seed, i, round).
+ * flb_keygen_gpu: Paillier::key_gen on the device — Philox candidates with the top two bits and
+ * bit 0 set, a small-prime sieve kernel, one Miller–Rabin round on every survivor and 39 more on
+ * the passers; the first two distinct probable primes (in candidate order) make the key, so the
+ * result is deterministic in seed (a different stream of primes from flb_keygen). */
+int flb_miller_rabin(const uint32_t* cand, uint32_t words, const uint32_t* mont_bases, uint32_t rounds,
+                     uint64_t seed, uint32_t* verdict, size_t count, void* stream);
+int flb_keygen_gpu(uint32_t key_bits, uint64_t seed, flb_pub** pub, flb_priv** priv, void* stream);
+
 /* ---------------------------------------------------------------- host-buffer pipeline (NEXT-1)
  * PAPER Fig. 4 / §V-A (L288–L298): host data -> compression -> copy to GPU -> HE -> copy back.
  * These take HOST pointers (pageable or pinned), split the batch into 32,768-element chunks and

@@ -56,6 +56,29 @@ def is_probable_prime(x: int, rng: random.Random, rounds: int = 40) -> bool:
     return True
 
 
+def miller_rabin_bases(x: int, bases: Iterable[int]) -> bool:
+    """Miller–Rabin with the given bases: True iff x passes every round.
+    Write x - 1 = d 2^s with d odd; x passes base a iff a^d = 1 or a^(d 2^r) = x - 1 for some
+    r < s (mod x).  A base with a mod x in {0} is treated as the round a^d mod x computes."""
+    if x < 3 or x % 2 == 0:
+        return x == 2
+    d, s = x - 1, 0
+    while d % 2 == 0:
+        d //= 2
+        s += 1
+    for a in bases:
+        y = pow(a, d, x)
+        if y == 1 or y == x - 1:
+            continue
+        for _ in range(s - 1):
+            y = y * y % x
+            if y == x - 1:
+                break
+        else:
+            return False
+    return True
+
+
 def random_prime(bits: int, rng: random.Random) -> int:
     """A random ``bits``-bit prime with its top two bits and its low bit set (reading c5)."""
     while True:

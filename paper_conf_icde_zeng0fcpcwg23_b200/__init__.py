@@ -22,7 +22,7 @@ from ._lib import LIB, FlbError, check
 __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
-    "Codec", "FlbError", "library_path", "op_cost", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
+    "Codec", "FlbError", "library_path", "op_cost", "keygen_gpu", "miller_rabin", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
     "reduce_segments_host",
 ]
 
@@ -112,6 +112,29 @@ def keygen(key_bits: int, seed: int) -> Tuple[PublicKey, PrivateKey]:
     check("flb_keygen", LIB.flb_keygen(key_bits, seed & 0xFFFFFFFFFFFFFFFF, ctypes.byref(pub), ctypes.byref(priv)))
     P = PublicKey(pub)
     return P, PrivateKey(priv, P)
+
+
+def keygen_gpu(key_bits: int, seed: int, stream=None) -> Tuple[PublicKey, PrivateKey]:
+    """Paillier::key_gen on the device: Philox candidates, sieve and Miller–Rabin kernels (PAPER L209)."""
+    pub, priv = ctypes.c_void_p(), ctypes.c_void_p()
+    check("flb_keygen_gpu", LIB.flb_keygen_gpu(key_bits, seed & 0xFFFFFFFFFFFFFFFF, ctypes.byref(pub), ctypes.byref(priv),
+                                               _stream(stream)))
+    P = PublicKey(pub)
+    return P, PrivateKey(priv, P)
+
+
+def miller_rabin(cand: torch.Tensor, rounds: int, mont_bases: Optional[torch.Tensor] = None, seed: int = 0,
+                 out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """Miller–Rabin verdicts (int32 [count], 1 = probable prime) for candidates [count, words]."""
+    words = cand.shape[1]
+    M = _check_batch(cand, words, "cand")
+    if mont_bases is not None:
+        _check_batch(mont_bases, words, "mont_bases")
+    if out is None:
+        out = torch.empty((M,), dtype=torch.int32, device=cand.device)
+    check("flb_miller_rabin", LIB.flb_miller_rabin(_ptr(cand), words, _ptr(mont_bases), rounds,
+                                                   seed & 0xFFFFFFFFFFFFFFFF, _ptr(out), M, _stream(stream)))
+    return out
 
 
 def key_from_primes(p: int, q: int) -> Tuple[PublicKey, PrivateKey]:

@@ -470,6 +470,31 @@ int run_modpow(const flb_pub* K, const uint32_t* dev, const uint32_t* sched, con
   return FLB_OK;
 }
 
+template <int X, int T>
+int run_mr(const uint32_t* cand, const uint32_t* bases, uint32_t rounds, uint64_t seed, uint64_t ctr0, uint32_t* verdict,
+           size_t count, int bw, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_miller_rabin<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)(1u << bw) * G * X * T * 4, st);
+  if (rc) return rc;
+  flb::MrArgs A;
+  A.cand = cand;
+  A.bases = bases;
+  A.rounds = rounds;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.verdict = verdict;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  A.bw = bw;
+  flb::k_miller_rabin<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
 template <int X, int T, bool DEBUG>
 int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
             cudaStream_t st) {
@@ -953,6 +978,110 @@ int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out
   } catch (const std::exception& ex) {
     return fail(FLB_EINVAL, ex.what());
   }
+}
+
+static int frame_key(uint32_t words, uint32_t* key) {
+  switch (words) {
+    case 32: *key = 512; return FLB_OK;
+    case 64: *key = 1024; return FLB_OK;
+    case 96: *key = 1536; return FLB_OK;
+    case 128: *key = 2048; return FLB_OK;
+    case 192: *key = 3072; return FLB_OK;
+    case 256: *key = 4096; return FLB_OK;
+  }
+  return fail(FLB_EINVAL, "words must be one of 32, 64, 96, 128, 192, 256");
+}
+
+int flb_miller_rabin(const uint32_t* cand, uint32_t words, const uint32_t* mont_bases, uint32_t rounds, uint64_t seed,
+                     uint32_t* verdict, size_t count, void* stream) {
+  if (!cand || !verdict || rounds == 0 || rounds > 64) return fail(FLB_EINVAL, "null pointer or rounds not in [1, 64]");
+  uint32_t key;
+  int rc = frame_key(words, &key);
+  if (rc) return rc;
+  if (count == 0) return FLB_OK;
+  const int bw = 5;
+  FLB_DISPATCH_ENC(key, run_mr, cand, mont_bases, rounds, seed, 0, verdict, count, bw, (cudaStream_t)stream);
+}
+
+int flb_keygen_gpu(uint32_t key_bits, uint64_t seed, flb_pub** pub, flb_priv** priv, void* stream) {
+  if (!pub || !priv) return fail(FLB_EINVAL, "null output pointer");
+  if (key_bits != 1024 && key_bits != 2048 && key_bits != 3072 && key_bits != 4096)
+    return fail(FLB_EINVAL, "key_bits must be 1024, 2048, 3072 or 4096");
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint32_t pbits = key_bits / 2, pwords = (pbits + 31) / 32;
+  uint32_t S = 32;
+  while (S < pwords) S += 32;
+  if (S == 160 || S == 224) S += 32;
+  uint32_t key;
+  int rc = frame_key(S, &key);
+  if (rc) return rc;
+  const uint64_t B = 8192;  // candidates per batch
+  std::vector<uint32_t> primes;
+  for (uint32_t p : H::small_primes()) primes.push_back(p);
+  uint32_t *d_cand = nullptr, *d_flag = nullptr, *d_primes = nullptr, *d_surv = nullptr, *d_ver = nullptr;
+  auto cleanup = [&] {
+    cudaFree(d_cand); cudaFree(d_flag); cudaFree(d_primes); cudaFree(d_surv); cudaFree(d_ver);
+  };
+  auto ck = [&](cudaError_t e, const char* what) {
+    if (e != cudaSuccess) {
+      g_err = std::string(what) + ": " + cudaGetErrorString(e);
+      cleanup();
+      return FLB_ECUDA;
+    }
+    return FLB_OK;
+  };
+  if ((rc = ck(cudaMalloc(&d_cand, B * S * 4), "cudaMalloc")) || (rc = ck(cudaMalloc(&d_flag, B * 4), "cudaMalloc")) ||
+      (rc = ck(cudaMalloc(&d_primes, primes.size() * 4), "cudaMalloc")) ||
+      (rc = ck(cudaMalloc(&d_surv, B * S * 4), "cudaMalloc")) || (rc = ck(cudaMalloc(&d_ver, B * 4), "cudaMalloc")))
+    return rc;
+  if ((rc = ck(cudaMemcpy(d_primes, primes.data(), primes.size() * 4, cudaMemcpyHostToDevice), "cudaMemcpy"))) return rc;
+  std::vector<uint32_t> flags(B), ver(B), host_c(B * S);
+  std::vector<Limbs> found;
+  for (uint64_t batch = 0; found.size() < 2 && batch < 4096; batch++) {
+    flb::k_gen_candidates<<<grid_1d(B * S), 256, 0, st>>>(d_cand, B, S, pbits, seed, batch * B);
+    flb::k_sieve<<<grid_1d(B), 256, 0, st>>>(d_cand, B, S, pwords, d_primes, (uint32_t)primes.size(), d_flag);
+    if ((rc = ck(cudaGetLastError(), "launch")) || (rc = ck(cudaMemcpyAsync(flags.data(), d_flag, B * 4,
+                                                                            cudaMemcpyDeviceToHost, st), "copy")) ||
+        (rc = ck(cudaMemcpyAsync(host_c.data(), d_cand, B * S * 4, cudaMemcpyDeviceToHost, st), "copy")) ||
+        (rc = ck(cudaStreamSynchronize(st), "sync")))
+      return rc;
+    std::vector<uint64_t> idx;
+    for (uint64_t i = 0; i < B; i++)
+      if (flags[i]) idx.push_back(i);
+    // round 1 on every sieve survivor, then 39 more on the passers (Miller–Rabin)
+    for (int phase = 0; phase < 2 && !idx.empty(); phase++) {
+      std::vector<uint32_t> surv(idx.size() * S);
+      for (size_t t = 0; t < idx.size(); t++)
+        std::memcpy(&surv[t * S], &host_c[idx[t] * S], S * 4);
+      if ((rc = ck(cudaMemcpyAsync(d_surv, surv.data(), surv.size() * 4, cudaMemcpyHostToDevice, st), "copy"))) return rc;
+      const uint32_t rounds = phase == 0 ? 1 : 39;
+      rc = flb_miller_rabin(d_surv, S, nullptr, rounds, seed ^ (0x4d52000000000000ull + batch * 2 + phase), d_ver,
+                            idx.size(), stream);
+      if (rc) { cleanup(); return rc; }
+      if ((rc = ck(cudaMemcpyAsync(ver.data(), d_ver, idx.size() * 4, cudaMemcpyDeviceToHost, st), "copy")) ||
+          (rc = ck(cudaStreamSynchronize(st), "sync")))
+        return rc;
+      std::vector<uint64_t> keep;
+      for (size_t t = 0; t < idx.size(); t++)
+        if (ver[t]) keep.push_back(idx[t]);
+      idx.swap(keep);
+    }
+    for (uint64_t i : idx) {
+      Limbs p(host_c.begin() + i * S, host_c.begin() + i * S + pwords);
+      if (found.empty() || H::cmp(found[0], p) != 0) found.push_back(p);
+      if (found.size() == 2) break;
+    }
+  }
+  cleanup();
+  if (found.size() < 2) return fail(FLB_EKEY, "no primes found");
+  try {
+    flb_priv* V = make_priv(found[0], found[1]);
+    *priv = V;
+    *pub = make_pub(V->pub->n);
+  } catch (const std::exception& ex) {
+    return fail(FLB_EKEY, ex.what());
+  }
+  return FLB_OK;
 }
 
 static int codec_args(const flb_pub* K, const flb_codec* cd, flb::CodecArgs* A) {

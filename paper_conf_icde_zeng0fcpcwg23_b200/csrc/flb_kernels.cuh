@@ -28,6 +28,14 @@ struct ModRef {
   uint32_t n0inv;     // -n^-1 mod 2^32 (reading c6)
 };
 
+// -n0^-1 mod 2^32 by Newton iteration (n0 odd)
+__device__ __forceinline__ uint32_t host_free_neg_inv32(uint32_t n0) {
+  uint32_t x = n0;
+#pragma unroll
+  for (int i = 0; i < 5; i++) x *= 2u - n0 * x;
+  return 0u - x;
+}
+
 // ----------------------------------------------------------------------------- group indexing
 template <int T>
 struct Grid {
@@ -382,6 +390,187 @@ __global__ void __launch_bounds__(32, FLB_MINB_ENC) k_modpow(const PowArgs A) {
 __global__ void k_fill_one(uint32_t* out, uint64_t count, uint32_t S) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count * S; i += (uint64_t)gridDim.x * blockDim.x)
     out[i] = (i % S) == 0 ? 1u : 0u;
+}
+
+// ----------------------------------------------------------------------------- Miller–Rabin (keygen)
+struct MrArgs {
+  const uint32_t* cand;       // [count][S] odd candidates >= 5
+  const uint32_t* bases;      // [count][rounds][S] Montgomery-form bases (< cand), or null: Philox
+  uint32_t rounds;
+  uint64_t seed, ctr0;
+  uint32_t* verdict;          // [count] 1 = passed every round
+  uint64_t count;
+  uint32_t* scratch;          // 2^bw * G * S
+  int bw;
+};
+
+// this group's exponent staging (S words): the candidate minus one, read bit-window by bit-window
+template <int X, int T>
+__device__ __forceinline__ uint32_t* exp_stage_group() {
+  constexpr int LD = X + 4;
+  __shared__ __align__(16) uint32_t ebuf[kMaxWarps * 32 * LD];
+  return ebuf + (threadIdx.x >> 5) * (32 * LD) + (int)(lane_id() & ~(uint32_t)(T - 1)) * LD;
+}
+
+template <int X>
+__device__ __forceinline__ uint32_t staged_word(const uint32_t* st, int w) {
+  return st[(w / X) * (X + 4) + (w % X)];
+}
+
+// group-wide equality of two distributed numbers
+template <int X, int T>
+__device__ __forceinline__ bool grp_equal(const uint32_t (&a)[X], const uint32_t (&b)[X]) {
+  uint32_t diff = 0;
+#pragma unroll
+  for (int j = 0; j < X; j++) diff |= a[j] ^ b[j];
+  const uint32_t bal = __ballot_sync(FULL, diff != 0);
+  const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
+  const uint32_t gm = (T == 32) ? 0xffffffffu : (((1u << T) - 1u) << base);
+  return (bal & gm) == 0;
+}
+
+// Miller–Rabin rounds for a batch of candidates, each with its own modulus.  Bases
+// are taken in Montgomery form (a random a~ < P is the Montgomery form of the random base
+// a = a~ R^-1 mod P), so no R^2 mod P is needed; x = a^d is formed by a fixed-window ladder over
+// the bits of d = (P-1)/2^s with warp-uniform control (zero digits and not-yet-started lanes
+// select instead of branching), then compared with 1 and P-1 after leaving the Montgomery domain.
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_ENC) k_miller_rabin(const MrArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  const int table = 1 << A.bw;
+  uint32_t* est = exp_stage_group<X, T>();
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t n[X], pm1[X], x[X], b[X], acc[X] = {}, y[X], one[X];
+    load_elem<X, T>(n, A.cand + e * S, S, valid);
+    if (!valid && g.k == 0) n[0] = 5;  // dummy modulus for idle groups
+    const uint32_t n0inv = __shfl_sync(FULL, host_free_neg_inv32(n[0]), 0, T);
+#pragma unroll
+    for (int j = 0; j < X; j++) pm1[j] = n[j];
+    if (g.k == 0) pm1[0] &= ~1u;  // P - 1 (P odd)
+    set_one<X, T>(one);
+    // s = trailing zeros of P - 1; bits(P - 1)
+    int lz = -1, hz = -1;
+#pragma unroll
+    for (int j = X - 1; j >= 0; j--) if (pm1[j]) lz = g.k * X * 32 + j * 32 + (__ffs(pm1[j]) - 1);
+#pragma unroll
+    for (int j = 0; j < X; j++) if (pm1[j]) hz = g.k * X * 32 + j * 32 + 31 - __clz(pm1[j]);
+    int s_bits = lz < 0 ? 0x7fffffff : lz;
+#pragma unroll
+    for (int o = 1; o < T; o <<= 1) s_bits = min(s_bits, __shfl_xor_sync(FULL, s_bits, o, T));
+    int top_bit = hz;
+#pragma unroll
+    for (int o = 1; o < T; o <<= 1) top_bit = max(top_bit, __shfl_xor_sync(FULL, top_bit, o, T));
+    const int dbits = top_bit + 1 - s_bits;  // bits of d
+    // stage P - 1 for digit extraction
+    __syncwarp();
+    {
+      uint4* q = reinterpret_cast<uint4*>(est + g.k * (X + 4));
+#pragma unroll
+      for (int v = 0; v < X / 4; v++) q[v] = make_uint4(pm1[4 * v], pm1[4 * v + 1], pm1[4 * v + 2], pm1[4 * v + 3]);
+    }
+    __syncwarp();
+    int topw = (dbits - 1) / A.bw;
+    topw = __reduce_max_sync(FULL, valid ? topw : 0);
+    int smax = __reduce_max_sync(FULL, valid ? s_bits : 1);
+    bool composite = false;
+#pragma unroll 1
+    for (uint32_t rd = 0; rd < A.rounds; rd++) {
+      if (A.bases) {
+        load_elem<X, T>(x, A.bases + (e * A.rounds + rd) * S, S, valid);
+      } else {
+        philox_r<X, T>(x, A.seed, (A.ctr0 + e) * 64 + rd, S, (uint32_t)(top_bit + 1));
+      }
+      // table: T[j] = x^j (Montgomery), j = 1 .. table-1
+      store_limbs<X>(tab + stride + g.k * X, x);
+#pragma unroll
+      for (int j = 0; j < X; j++) b[j] = x[j];
+#pragma unroll 1
+      for (int i = 2; i < table; i++) {
+        mont_mul<X, T>(b, b, x, n, n0inv);
+        store_limbs<X>(tab + (size_t)i * stride + g.k * X, b);
+      }
+      bool started = false;
+#pragma unroll 1
+      for (int w = topw; w >= 0; w--) {
+        if (w != topw) {
+#pragma unroll 1
+          for (int sq = 0; sq < A.bw; sq++) mont_sqr<X, T>(acc, acc, n, n0inv);
+        }
+        // digit w of d = bits [s + w bw, s + w bw + bw) of P - 1 (zero beyond d's top)
+        uint32_t dgt = 0;
+        if (w * A.bw < dbits) {
+          const int lo = s_bits + w * A.bw, word = lo >> 5, off = lo & 31;
+          uint32_t v = staged_word<X>(est, word) >> off;
+          if (off + A.bw > 32 && word + 1 < S) v |= staged_word<X>(est, word + 1) << (32 - off);
+          const int nb = min(A.bw, dbits - w * A.bw);
+          dgt = v & ((1u << nb) - 1u);
+        }
+        load_limbs_plain<X>(b, tab + (size_t)(dgt ? dgt : 1u) * stride + g.k * X);
+        mont_mul<X, T>(y, acc, b, n, n0inv);
+#pragma unroll
+        for (int j = 0; j < X; j++) acc[j] = dgt ? (started ? y[j] : b[j]) : acc[j];
+        started = started || (dgt != 0);
+      }
+      mont_mul<X, T>(y, acc, one, n, n0inv);  // a^d mod P
+      // every lane evaluates every comparison (ballots must never sit in divergent code)
+      const bool eq1 = grp_equal<X, T>(y, one), eqm1 = grp_equal<X, T>(y, pm1);
+      bool pass = eq1 || eqm1;
+#pragma unroll 1
+      for (int r = 1; r < smax; r++) {
+        mont_sqr<X, T>(acc, acc, n, n0inv);
+        mont_mul<X, T>(y, acc, one, n, n0inv);
+        const bool eq = grp_equal<X, T>(y, pm1);
+        pass = pass || (r < s_bits && eq);
+      }
+      composite = composite || !pass;
+    }
+    if (valid && g.k == 0) A.verdict[e] = composite ? 0u : 1u;
+  }
+}
+
+// candidates for key generation: Philox words, bits above `bits` cleared, top two bits and bit 0
+// set (reading c5), limbs above the prime's words zero; one thread per limb.
+__global__ void k_gen_candidates(uint32_t* cand, uint64_t count, uint32_t S, uint32_t bits, uint64_t seed,
+                                 uint64_t ctr0) {
+  const uint64_t total = count * S;
+  for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < total; t += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t i = t / S;
+    const uint32_t w = (uint32_t)(t - i * S);
+    uint32_t v = 0;
+    if (32u * w < bits) {
+      const uint64_t idx = ctr0 + i;
+      const uint4 o = philox4x32_10(make_uint4((uint32_t)idx, (uint32_t)(idx >> 32), w / 4, 0x6b657967u),
+                                    make_uint2((uint32_t)seed, (uint32_t)(seed >> 32)));
+      v = (&o.x)[w & 3];
+      if (32u * (w + 1) > bits) v &= (1u << (bits - 32u * w)) - 1u;
+      const uint32_t top = bits - 1;
+      if (w == top / 32) v |= 1u << (top % 32);
+      if (w == (top - 1) / 32) v |= 1u << ((top - 1) % 32);
+      if (w == 0) v |= 1u;
+    }
+    cand[t] = v;
+  }
+}
+
+// small-prime sieve: flag[i] = 1 if no prime in `primes` divides candidate i
+__global__ void k_sieve(const uint32_t* __restrict__ cand, uint64_t count, uint32_t S, uint32_t words,
+                        const uint32_t* __restrict__ primes, uint32_t nprimes, uint32_t* __restrict__ flag) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t* c = cand + i * S;
+    uint32_t ok = 1;
+    for (uint32_t k = 0; k < nprimes && ok; k++) {
+      const uint32_t p = __ldg(primes + k);
+      uint64_t r = 0;
+      for (int w = (int)words - 1; w >= 0; w--) r = ((r << 32) | c[w]) % p;
+      ok = r != 0;
+    }
+    flag[i] = ok;
+  }
 }
 
 // ----------------------------------------------------------------------------- hom-add

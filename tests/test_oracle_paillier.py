@@ -220,3 +220,19 @@ def test_draw_r_range_and_determinism():
     ptoy, qtoy = KEYS["toy16"]
     for i in range(50):
         assert 1 <= philox.draw_r(ptoy * qtoy, 9, i, 32) < (1 << 15)
+
+
+def test_miller_rabin_with_given_bases():
+    # primes pass every base; composites are caught by some base; base 2 alone is fooled by the
+    # strong pseudoprime 2047 = 23 * 89 (a textbook fact), bases 2 and 3 by 1373653 = 829 * 1657
+    for pr in (3, 5, 7, 101, 7919, (1 << 61) - 1, (1 << 89) - 1):
+        assert paillier.miller_rabin_bases(pr, [b for b in (2, 3, 5, 7, 11) if b < pr - 1] + [pr - 1])
+    assert paillier.miller_rabin_bases(2047, [2]) and not paillier.miller_rabin_bases(2047, [3])
+    assert paillier.miller_rabin_bases(1373653, [2, 3]) and not paillier.miller_rabin_bases(1373653, [5])
+    for c in (561, 1105, 1729, 2465, 2821, 6601, 8911):  # Carmichael numbers: base 2 catches them
+        assert not paillier.miller_rabin_bases(c, [2])
+    rng = random.Random(8)
+    for _ in range(300):  # agreement with trial division on random odd 20-bit numbers, 8 random bases
+        x = rng.randrange(3, 1 << 20) | 1
+        is_p = all(x % d for d in range(3, int(math.isqrt(x)) + 1, 2))
+        assert paillier.miller_rabin_bases(x, [rng.randrange(2, x - 1) for _ in range(8)]) == is_p
