@@ -300,10 +300,22 @@ __device__ __forceinline__ void mont_mul(uint32_t (&r)[X], const uint32_t (&a)[X
 
 // r = a * a * R^-1 mod N
 template <int X, int T>
+__device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
+                                                uint32_t n0inv);
+
+#ifndef FLB_SQR_BLOCKS
+#define FLB_SQR_BLOCKS 0  // measured slower on B200; kept as a parity-tested experiment
+#endif
+
+template <int X, int T>
 __device__ __forceinline__ void mont_sqr(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
                                          uint32_t n0inv) {
-  stage<X, T>(a);
-  mont_mul_staged<X, T>(r, a, n, n0inv);
+  if constexpr (FLB_SQR_BLOCKS && T >= 4) {
+    mont_sqr_blocks<X, T>(r, a, n, n0inv);
+  } else {
+    stage<X, T>(a);
+    mont_mul_staged<X, T>(r, a, n, n0inv);
+  }
 }
 
 // r = a * b mod 2^(32*S) (the low half of the plain product).
@@ -358,6 +370,190 @@ __device__ __forceinline__ void mul_full(uint32_t (&lo)[X], uint32_t (&hi)[X], c
 #pragma unroll
   for (int t = 0; t < X; t++) lo[t] = res[t];
   collapse<X, T>(hi, E, O, pend);
+}
+
+// ----------------------------------------------------------------------------- squaring
+// Montgomery squaring with the square computed by lane-local X x X block products (PAPER L207:
+// squarings are ~87 % of a modexp's multiplications).  a^2 = sum_k A_k^2 2^(2 k X w) +
+// 2 sum_{k<l} A_k A_l 2^((k+l) X w), A_k = lane k's chunk.  Lane k computes its square block and
+// the cross blocks (k, k+d mod T) for d = 1 .. T/2-1, plus d = T/2 when k < T/2 — every
+// unordered pair exactly once, T/2 + 1 blocks per lane (vs T rows of CIOS products): 1280 instead
+// of 2048 limb products per lane at T = 8.  Blocks are summed (cross blocks doubled) into 64-bit
+// column sums in shared memory — two non-overlapping write phases per block round, no atomics —
+// then one carry normalisation gives t = a^2 as (t_lo, t_hi) in the CIOS layout, and a reduce-only
+// CIOS pass gives REDC(t_lo) + t_hi = a^2 R^-1 (mod N), < 2N, canonicalised.
+
+// lane-local product row: acc += a * bi (no neighbour lanes), shift one word, return the word out
+template <int X>
+__device__ __forceinline__ uint32_t local_row(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
+                                              const uint32_t (&a)[X], uint32_t bi) {
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
+  chain_odd<X, true>(O, a, bi);
+  chain_even<X>(E, a, bi);
+  const uint32_t out = E[0];
+  pend = E[1];
+  uint32_t nE[X + 1], nO[X + 1];
+#pragma unroll
+  for (int t = 0; t <= X; t++) nE[t] = O[t];
+#pragma unroll
+  for (int t = 0; t + 2 <= X; t++) nO[t] = E[t + 2];
+  nO[X - 1] = 0;
+  nO[X] = 0;
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
+  return out;
+}
+
+// per-group 64-bit column sums for the 2S-word square
+template <int X, int T>
+__device__ __forceinline__ unsigned long long* col_group() {
+  constexpr int S = X * T;
+  __shared__ __align__(16) unsigned long long cbuf[kMaxWarps * 32 / T * 2 * S];
+  return cbuf + ((threadIdx.x >> 5) * (32 / T) + (int)((lane_id() & 31u) / T)) * (2 * S);
+}
+
+// reduce-only CIOS step: m = word0 * n0inv; acc += m N; acc >>= 32
+template <int X, int T>
+__device__ __forceinline__ void redc_step(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
+                                          const uint32_t (&n)[X], uint32_t n0inv) {
+  const int k = (int)(lane_id() & (T - 1));
+  // merge the pending word into word 0; its carry enters the O chain (word 1) after m is formed
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
+  const uint32_t m = __shfl_sync(FULL, E[0], 0, T) * n0inv;
+  chain_odd<X, true>(O, n, m);
+  chain_even<X>(E, n, m);
+  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
+  if (k == T - 1) up = 0;
+  pend = E[1];
+  uint32_t nE[X + 1], nO[X + 1];
+#pragma unroll
+  for (int t = 0; t <= X; t++) nE[t] = O[t];
+#pragma unroll
+  for (int t = 0; t + 2 <= X; t++) nO[t] = E[t + 2];
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[X - 2]) : "r"(up));
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[X - 1]));
+  nO[X] = 0;
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
+}
+
+template <int X, int T>
+__device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
+                                                uint32_t n0inv) {
+  constexpr int LD = X + 4, S = X * T, NB = T / 2 + 1;
+  static_assert(T >= 4, "block squaring needs at least 4 lanes per integer");
+  const int k = (int)(lane_id() & (T - 1));
+  stage<X, T>(a);
+  const uint32_t* bs = stage_group<X, T>();
+  unsigned long long* col = col_group<X, T>();
+#pragma unroll
+  for (int j = 0; j < 2 * X; j += 2)
+    *reinterpret_cast<ulonglong2*>(col + 2 * X * k + j) = make_ulonglong2(0ull, 0ull);
+  __syncwarp();
+#pragma unroll 1
+  for (int blk = 0; blk < NB; blk++) {
+    const int l = (k + blk) & (T - 1);
+    const bool active = (blk < T / 2) || (k < T / 2);
+    const bool wraps = (k + blk) >= T;
+    const unsigned long long f = blk == 0 ? 1ull : 2ull;
+    const uint32_t* row = bs + l * LD;
+    uint32_t E[X + 1], O[X + 1], pend = 0, lo[X], hi[X];
+#pragma unroll
+    for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
+#pragma unroll
+    for (int jj = 0; jj < X; jj++) lo[jj] = local_row<X>(E, O, pend, a, row[jj]);
+    // the high X words (the block product is < 2^(64 X): nothing above)
+    asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(hi[0]) : "r"(E[0]), "r"(pend));
+#pragma unroll
+    for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(hi[t]) : "r"(E[t]), "r"(O[t - 1]));
+    unsigned long long* cb = col + X * (k + l);
+    // f * (lo, hi) into the column sums: batches of 8 columns, all loads of a batch before its
+    // stores (ptxas would otherwise serialise each load behind the previous store)
+    const unsigned sh = blk == 0 ? 0u : 1u;
+#pragma unroll
+    for (int ph = 0; ph < 2; ph++) {
+      if (active && (wraps == (ph == 1))) {
+#pragma unroll
+        for (int j0 = 0; j0 < 2 * X; j0 += 8) {
+          ulonglong2 v[4];
+#pragma unroll
+          for (int u = 0; u < 4; u++) v[u] = *reinterpret_cast<const ulonglong2*>(cb + j0 + 2 * u);
+#pragma unroll
+          for (int u = 0; u < 4; u++) {
+            const int j = j0 + 2 * u;
+            const uint32_t w0 = j < X ? lo[j] : hi[j - X], w1 = j + 1 < X ? lo[j + 1] : hi[j + 1 - X];
+            v[u].x += (unsigned long long)w0 << sh;
+            v[u].y += (unsigned long long)w1 << sh;
+          }
+#pragma unroll
+          for (int u = 0; u < 4; u++) *reinterpret_cast<ulonglong2*>(cb + j0 + 2 * u) = v[u];
+        }
+      }
+      __syncwarp();
+    }
+    (void)f;
+  }
+  // normalise lane k's two chunks: lo = columns [kX, kX+X), hi = [S + kX, S + kX + X)
+  uint32_t tl[X], th[X];
+  unsigned long long cl = 0, ch = 0;
+  {
+    const unsigned long long* pl = col + X * k;
+    const unsigned long long* ph = col + S + X * k;
+#pragma unroll
+    for (int j = 0; j < X; j++) {
+      cl += pl[j];
+      tl[j] = (uint32_t)cl;
+      cl >>= 32;
+      ch += ph[j];
+      th[j] = (uint32_t)ch;
+      ch >>= 32;
+    }
+  }
+  // chunk chain lo_0 .. lo_{T-1}, hi_0 .. hi_{T-1}: pass each chunk's carry to the next chunk
+  uint32_t inl_lo = __shfl_up_sync(FULL, (uint32_t)cl, 1, T), inl_hi = __shfl_up_sync(FULL, (uint32_t)(cl >> 32), 1, T);
+  uint32_t inh_lo = __shfl_up_sync(FULL, (uint32_t)ch, 1, T), inh_hi = __shfl_up_sync(FULL, (uint32_t)(ch >> 32), 1, T);
+  const uint32_t top_lo = __shfl_sync(FULL, (uint32_t)cl, T - 1, T), top_hi = __shfl_sync(FULL, (uint32_t)(cl >> 32), T - 1, T);
+  if (k == 0) {
+    inl_lo = 0; inl_hi = 0;
+    inh_lo = top_lo; inh_hi = top_hi;
+  }
+  uint32_t gl, gh;
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(tl[0]) : "r"(inl_lo));
+  asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(tl[1]) : "r"(inl_hi));
+#pragma unroll
+  for (int t = 2; t < X; t++) asm volatile("addc.cc.u32 %0, %0, 0;" : "+r"(tl[t]));
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(gl));
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(th[0]) : "r"(inh_lo));
+  asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(th[1]) : "r"(inh_hi));
+#pragma unroll
+  for (int t = 2; t < X; t++) asm volatile("addc.cc.u32 %0, %0, 0;" : "+r"(th[t]));
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(gh));
+  {
+    // single-bit carries along the 2T-chunk chain (lookahead over both ballots)
+    const uint32_t GL = __ballot_sync(FULL, gl != 0), PL = __ballot_sync(FULL, all_ones<X>(tl));
+    const uint32_t GH = __ballot_sync(FULL, gh != 0), PH = __ballot_sync(FULL, all_ones<X>(th));
+    const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
+    const uint64_t mask = (T == 32) ? 0xffffffffull : ((1ull << T) - 1);
+    const uint64_t gg = (((uint64_t)GL >> base) & mask) | ((((uint64_t)GH >> base) & mask) << T);
+    const uint64_t pp = (((uint64_t)PL >> base) & mask) | ((((uint64_t)PH >> base) & mask) << T);
+    const uint64_t c = ((pp | gg) + gg) ^ pp;
+    add_word_propagate<X>(tl, (uint32_t)((c >> k) & 1u));
+    add_word_propagate<X>(th, (uint32_t)((c >> (T + k)) & 1u));
+  }
+  // REDC(t_lo) + t_hi
+  uint32_t E[X + 1], O[X + 1], pend = 0;
+#pragma unroll
+  for (int t = 0; t < X; t++) { E[t] = tl[t]; O[t] = 0; }
+  E[X] = 0;
+  O[X] = 0;
+#pragma unroll 1
+  for (int kk = 0; kk < T; kk++) {
+#pragma unroll
+    for (int jj = 0; jj < X; jj++) redc_step<X, T>(E, O, pend, n, n0inv);
+  }
+  const uint32_t over1 = collapse<X, T>(r, E, O, pend);
+  const uint32_t over2 = grp_add<X, T>(r, r, th);
+  grp_cond_sub<X, T>(r, n, over1 | over2);
 }
 
 // ----------------------------------------------------------------------------- loads / stores

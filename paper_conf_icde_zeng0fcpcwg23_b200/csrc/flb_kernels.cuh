@@ -147,11 +147,10 @@ __device__ __forceinline__ void modexp_sched(uint32_t (&acc)[X], uint32_t (&x)[X
     for (int i = 0; i < steps; i++) {
       if (i == sq) {
         load_limbs_plain<X>(b, tab + (size_t)idx * stride + k * X);
-        stage<X, T>(b);
+        mont_mul<X, T>(acc, acc, b, n, n0inv);
       } else {
-        stage<X, T>(acc);
+        mont_sqr<X, T>(acc, acc, n, n0inv);
       }
-      mont_mul_staged<X, T>(acc, acc, n, n0inv);
     }
   }
 }

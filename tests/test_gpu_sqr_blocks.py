@@ -1,0 +1,22 @@
+"""The block-squaring experiment (FLB_SQR_BLOCKS=1 build) stays bit-exact: run the
+parity suite's encrypt/decrypt cases against a library built with it, when that build exists."""
+
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+VARIANT = os.path.join(ROOT, "build_variants", "sq.so")
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.skipif(not os.path.exists(VARIANT), reason="FLB_SQR_BLOCKS=1 variant not built")
+def test_block_squaring_variant_parity():
+    env = dict(os.environ, FLB_LIB_PATH=VARIANT)
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "tests/test_gpu_parity.py",
+                        "-k", "encrypt or decrypt or scalar"], cwd=ROOT, env=env, capture_output=True, text=True,
+                       timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
