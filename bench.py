@@ -405,11 +405,10 @@ def run_flb(args):
         def e2e_step(s):
             nonlocal h2d, d2h
             h2d = d2h = 0
-            for c in range(CLIENTS):
-                flb.pack_encrypt_host(pub, cd, grads_np[c], seed=3000 + s, ctr0=(rank * CLIENTS + c) * rows,
-                                      priv=kh, out=cts_h[c * rows:(c + 1) * rows])
-                h2d += grads_np[c].nbytes
-                d2h += rows * ctw * 4
+            flb.pack_encrypt_host_multi(pub, cd, grads_np, seed=3000 + s, ctr0=rank * CLIENTS * rows, priv=kh,
+                                        out=cts_h)
+            h2d += sum(g.nbytes for g in grads_np)
+            d2h += cts_h.nbytes
             part_h = flb.reduce_segments_host(pub, cts_h, offs_np, idx_np, max_segment_len=CLIENTS)
             h2d += cts_h.nbytes + offs_np.nbytes + idx_np.nbytes
             d2h += part_h.nbytes
@@ -444,7 +443,7 @@ def run_flb(args):
             e_ms, h2d, d2h = float(tm[0]), float(t[1]), float(t[2])
         e2e = {"value": total_ops / (e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": e_ms,
-               "path": "C-ABI host-buffer pipeline: flb_pack_encrypt_host x %d clients -> flb_reduce_segments_host "
+               "path": "C-ABI host-buffer pipeline: flb_pack_encrypt_host_multi (%d clients) -> flb_reduce_segments_host "
                        "-> %sflb_decrypt_unpack_host; host wall clock per step" %
                        (CLIENTS, "NCCL all_to_all + finish -> " if world > 1 else "")}
 

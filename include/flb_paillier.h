@@ -212,6 +212,15 @@ int flb_pack_encrypt_host(const flb_pub* pub, const flb_priv* priv, const flb_co
                           const float* x_host, size_t n_values, uint64_t seed, uint64_t ctr0,
                           uint32_t* c_host);
 
+/* ①–④ for several value arrays at once (e.g. the gradients of several clients): array a is packed
+ * into its own ceil(n_values[a]/slots) plaintexts (its own slot alignment) and all plaintexts are
+ * encrypted as one batch, in array order, with counter ctr0 + global plaintext index; c_host
+ * receives sum_a ceil(n_values[a]/slots) ciphertexts.  Same bits as one flb_pack_encrypt_host call
+ * per array with the matching ctr0. */
+int flb_pack_encrypt_host_multi(const flb_pub* pub, const flb_priv* priv, const flb_codec* codec,
+                                const float* const* x_hosts, const size_t* n_values, size_t n_arrays,
+                                uint64_t seed, uint64_t ctr0, uint32_t* c_host);
+
 /* ⑤–⑨: c_host [ceil(n_values/slots)][ct_words] -> decrypt -> unpack + dequantise -> x_host
  * float32 [n_values]; summands_host: uint32 [ceil(n_values/slots)] or NULL (then
  * summands_scalar).  pub must be priv's public key.  Errors: FLB_EINVAL, FLB_ECUDA. */

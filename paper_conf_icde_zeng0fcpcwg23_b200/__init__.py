@@ -23,7 +23,7 @@ __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
     "Codec", "FlbError", "library_path", "op_cost", "keygen_gpu", "miller_rabin", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
-    "reduce_segments_host",
+    "reduce_segments_host", "pack_encrypt_host_multi",
 ]
 
 library_path = _lib.LIB_PATH
@@ -363,6 +363,25 @@ def pack_encrypt_host(pub: PublicKey, codec: Codec, x, seed: int = 0, ctr0: int 
     check("flb_pack_encrypt_host", LIB.flb_pack_encrypt_host(pub.handle, priv.handle if priv else None,
                                                              ctypes.byref(cs), _np_ptr(x), x.shape[0],
                                                              seed & 0xFFFFFFFFFFFFFFFF, ctr0, _np_ptr(out)))
+    return out
+
+
+def pack_encrypt_host_multi(pub: PublicKey, codec: Codec, xs, seed: int = 0, ctr0: int = 0,
+                            priv: Optional[PrivateKey] = None, out=None):
+    """Several host float32 arrays (e.g. one per client), each packed with its own slot alignment,
+    encrypted as one pipelined batch -> host ciphertexts [sum_a ceil(len_a/S), ct_words]."""
+    import numpy as np
+    xs = [np.ascontiguousarray(x, dtype=np.float32) for x in xs]
+    M = sum(codec.num_plaintexts(x.shape[0]) for x in xs)
+    if out is None:
+        out = np.empty((M, pub.ct_words), dtype=np.uint32)
+    ptrs = (ctypes.c_void_p * len(xs))(*[x.ctypes.data for x in xs])
+    lens = (ctypes.c_size_t * len(xs))(*[x.shape[0] for x in xs])
+    cs = codec.struct()
+    check("flb_pack_encrypt_host_multi", LIB.flb_pack_encrypt_host_multi(pub.handle, priv.handle if priv else None,
+                                                                         ctypes.byref(cs), ptrs, lens, len(xs),
+                                                                         seed & 0xFFFFFFFFFFFFFFFF, ctr0,
+                                                                         _np_ptr(out)))
     return out
 
 

@@ -64,6 +64,8 @@ SIGNATURES = {
     "flb_miller_rabin": (ctypes.c_int, [_P, _U32, _P, _U32, _U64, _P, _SZ, _P]),
     "flb_keygen_gpu": (ctypes.c_int, [_U32, _U64, ctypes.POINTER(_P), ctypes.POINTER(_P), _P]),
     "flb_pack_encrypt_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _U64, _U64, _P]),
+    "flb_pack_encrypt_host_multi": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _P, _SZ, _U64, _U64,
+                                                    _P]),
     "flb_decrypt_unpack_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P]),
     "flb_reduce_segments_host": (ctypes.c_int, [_P, _P, _SZ, _P, _P, _SZ, _SZ, _P]),
     "flb_op_cost": (ctypes.c_int, [_P, _P, ctypes.c_int, ctypes.POINTER(_U64), ctypes.POINTER(_U64)]),

@@ -158,6 +158,76 @@ int flb_pack_encrypt_host(const flb_pub* pub, const flb_priv* priv, const flb_co
   return FLB_OK;
 }
 
+int flb_pack_encrypt_host_multi(const flb_pub* pub, const flb_priv* priv, const flb_codec* codec,
+                                const float* const* x_hosts, const size_t* n_values, size_t n_arrays, uint64_t seed,
+                                uint64_t ctr0, uint32_t* c_host) {
+  if (!pub || !codec || !x_hosts || !n_values || !c_host || codec->slots == 0) {
+    g_perr = "null pointer or zero slots";
+    return FLB_EINVAL;
+  }
+  if (n_arrays == 0) return FLB_OK;
+  DevCtx* C;
+  RC(ctx_for_device(&C));
+  std::lock_guard<std::mutex> lk(C->mu);
+  const size_t S = codec->slots, ptw = flb_pt_words(pub), ctw = flb_ct_words(pub);
+  size_t total_v = 0, total_pt = 0;
+  for (size_t a = 0; a < n_arrays; a++) {
+    if (n_values[a] && !x_hosts[a]) {
+      g_perr = "null array";
+      return FLB_EINVAL;
+    }
+    total_v += n_values[a];
+    total_pt += (n_values[a] + S - 1) / S;
+  }
+  if (total_pt == 0) return FLB_OK;
+  // all values in (pinned staging, one H2D per array on stream 0), every array packed into its own
+  // plaintexts (slot alignment per array), then encryption in chunks with D2H overlap on 2 streams
+  RC(ensure_host(C->pin_aux[0], total_v * 4 + 16));
+  RC(ensure_dev(C->d_aux[0], total_v * 4 + 16));
+  RC(ensure_dev(C->d_mid[0], total_pt * ptw * 4));
+  for (int s = 0; s < 2; s++) {
+    RC(ensure_host(C->pin_out[s], kChunkPt * ctw * 4));
+    RC(ensure_dev(C->d_out[s], kChunkPt * ctw * 4));
+  }
+  size_t v0 = 0, p0 = 0;
+  for (size_t a = 0; a < n_arrays; a++) {
+    if (!n_values[a]) continue;
+    std::memcpy((float*)C->pin_aux[0].p + v0, x_hosts[a], n_values[a] * 4);
+    PCK(cudaMemcpyAsync((float*)C->d_aux[0].p + v0, (float*)C->pin_aux[0].p + v0, n_values[a] * 4,
+                        cudaMemcpyHostToDevice, C->st[0]));
+    int rc = flb_pack(pub, codec, (const float*)C->d_aux[0].p + v0, n_values[a], (uint32_t*)C->d_mid[0].p + p0 * ptw,
+                      C->st[0]);
+    if (rc) return lib_err(rc, "flb_pack");
+    v0 += n_values[a];
+    p0 += (n_values[a] + S - 1) / S;
+  }
+  PCK(cudaEventRecord(C->done[0], C->st[0]));
+  PCK(cudaStreamWaitEvent(C->st[1], C->done[0], 0));
+  const size_t chunks = (total_pt + kChunkPt - 1) / kChunkPt;
+  size_t pending_pt0 = 0, pending_n = 0;
+  int pending_s = -1;
+  for (size_t i = 0; i < chunks; i++) {
+    const int s = (int)(i & 1);
+    const size_t pt0 = i * kChunkPt, npt = std::min(kChunkPt, total_pt - pt0);
+    const uint32_t* src = (const uint32_t*)C->d_mid[0].p + pt0 * ptw;
+    int rc = priv ? flb_encrypt_crt(priv, src, nullptr, seed, ctr0 + pt0, (uint32_t*)C->d_out[s].p, npt, C->st[s])
+                  : flb_encrypt(pub, src, nullptr, seed, ctr0 + pt0, (uint32_t*)C->d_out[s].p, npt, C->st[s]);
+    if (rc) return lib_err(rc, "flb_encrypt");
+    PCK(cudaMemcpyAsync(C->pin_out[s].p, C->d_out[s].p, npt * ctw * 4, cudaMemcpyDeviceToHost, C->st[s]));
+    PCK(cudaEventRecord(C->done[s], C->st[s]));
+    if (pending_s >= 0) {
+      PCK(cudaEventSynchronize(C->done[pending_s]));
+      std::memcpy(c_host + pending_pt0 * ctw, C->pin_out[pending_s].p, pending_n * ctw * 4);
+    }
+    pending_s = s;
+    pending_pt0 = pt0;
+    pending_n = npt;
+  }
+  PCK(cudaEventSynchronize(C->done[pending_s]));
+  std::memcpy(c_host + pending_pt0 * ctw, C->pin_out[pending_s].p, pending_n * ctw * 4);
+  return FLB_OK;
+}
+
 int flb_decrypt_unpack_host(const flb_priv* priv, const flb_pub* pub, const flb_codec* codec,
                             const uint32_t* c_host, size_t n_values, const uint32_t* summands_host,
                             uint32_t summands_scalar, float* x_host) {

@@ -58,3 +58,17 @@ def test_decrypt_unpack_host_per_plaintext_counts():
     cnt = np.ones(c.shape[0], dtype=np.uint32)
     out = flb.decrypt_unpack_host(priv, cd, c, x.shape[0], summands=cnt)
     assert np.max(np.abs(out - x)) <= 1.0 / ((1 << 44) - 1) + np.abs(x).max() * 2 ** -24
+
+
+def test_multi_array_host_encrypt_equals_per_array_calls():
+    p, q = golden_keys()["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    cd = flb.Codec(1.0, 29, 3, 31)
+    xs = [synthetic.c2_gradient(c, n=n) for c, n in enumerate([31 * 40000 + 5, 17, 31 * 3000, 0, 999])]
+    multi = flb.pack_encrypt_host_multi(pub, cd, xs, seed=21, ctr0=100, priv=priv)
+    parts, ctr = [], 100
+    for x in xs:
+        if x.shape[0]:
+            parts.append(flb.pack_encrypt_host(pub, cd, x, seed=21, ctr0=ctr, priv=priv))
+            ctr += cd.num_plaintexts(x.shape[0])
+    assert np.array_equal(multi, np.concatenate(parts))
