@@ -13,7 +13,19 @@ VARIANT = os.path.join(ROOT, "build_variants", "sq.so")
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.skipif(not os.path.exists(VARIANT), reason="FLB_SQR_BLOCKS=1 variant not built")
+def _variant_current():
+    """The variant exists and is newer than every source it is built from (else it is stale)."""
+    if not os.path.exists(VARIANT):
+        return False
+    sys.path.insert(0, os.path.join(ROOT, "paper_conf_icde_zeng0fcpcwg23_b200"))
+    import build  # noqa: E402
+    t = os.path.getmtime(VARIANT)
+    return all(os.path.getmtime(d) <= t for d in build.deps())
+
+
+@pytest.mark.skipif(not _variant_current(), reason="FLB_SQR_BLOCKS=1 variant not built or stale "
+                    "(FLB_LIB_PATH=build_variants/sq.so FLB_NVCC_EXTRA=-DFLB_SQR_BLOCKS=1 python "
+                    "paper_conf_icde_zeng0fcpcwg23_b200/build.py --force)")
 def test_block_squaring_variant_parity():
     env = dict(os.environ, FLB_LIB_PATH=VARIANT)
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "tests/test_gpu_parity.py",
