@@ -114,14 +114,26 @@ int flb_scalar_mul(const flb_pub* pub, const uint32_t* c, const uint32_t* e, uin
 
 /* Segmented ciphertext product (Fig. 2 server aggregation; repeated Eq. 5):
  * out_j = prod_{t = offsets[j]}^{offsets[j+1]-1} c[idx ? idx[t] : t] mod n^2, out_j = 1 for an
- * empty segment.  c: [num_inputs][ct_words]; idx: device int64 [offsets[num_segments]] or
- * NULL; offsets: device int64 [num_segments+1], non-decreasing, offsets[0] = 0.
- * max_segment_len: an upper bound on any segment's length if known (sizes the number of
- * reduction levels), 0 = unknown (num_inputs is used).  out: [num_segments][ct_words], must not
- * alias c.  Errors: FLB_EINVAL, FLB_ECUDA. */
+ * empty segment.  c: [num_inputs][ct_words]; idx: device int64 [num_entries] (entries may repeat
+ * inputs) or NULL (then entry t is input t and num_entries <= num_inputs); offsets: device int64
+ * [num_segments+1], non-decreasing, offsets[0] = 0, offsets[num_segments] = num_entries (host
+ * value passed in num_entries, it sizes the scratch).  max_segment_len: an upper bound on any
+ * segment's length if known (sizes the number of reduction levels), 0 = unknown (num_entries).
+ * out: [num_segments][ct_words], must not alias c.  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_reduce_segments(const flb_pub* pub, const uint32_t* c, size_t num_inputs,
-                        const int64_t* idx, const int64_t* offsets, size_t num_segments,
-                        size_t max_segment_len, uint32_t* out, void* stream);
+                        const int64_t* idx, size_t num_entries, const int64_t* offsets,
+                        size_t num_segments, size_t max_segment_len, uint32_t* out, void* stream);
+
+/* Segmented multi-exponentiation: out_j = prod_{t = offsets[j]}^{offsets[j+1]-1} c[idx ? idx[t] : t]^(e_t)
+ * mod n^2 = E(sum_t e_t m_t) — Hetero-LR's per-feature sum of encrypted residuals x feature values
+ * (PAPER L375 models; Table I mod_pow, L246, composed with Eq. 5).  e: device [num_entries][e_words]
+ * (1 <= e_words <= 8), one exponent per entry; num_entries = offsets[num_segments].  Long segments
+ * use Pippenger's bucket method (digit buckets and bit-plane products are segmented products);
+ * short ones scalar-mul + product.  Results are identical either way.  Scratch ~ (num_entries * W * 8
+ * + buckets * ct_words * 4) bytes from the stream-ordered pool.  Errors: FLB_EINVAL, FLB_ECUDA. */
+int flb_multiexp_segments(const flb_pub* pub, const uint32_t* c, size_t num_inputs, const int64_t* idx,
+                          const uint32_t* e, uint32_t e_words, const int64_t* offsets,
+                          size_t num_segments, size_t num_entries, uint32_t* out, void* stream);
 
 /* Encoding-quantisation + batch compression parameters (PAPER §IV-B/§IV-C):
  * alpha: gradient bound (Eq. 6), qbits: r of Eq. 7 (L221, 1..52), pad_bits: b of Eq. 8

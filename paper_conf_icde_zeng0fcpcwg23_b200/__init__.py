@@ -21,7 +21,7 @@ from ._lib import LIB, FlbError, check
 
 __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
-    "scalar_mul", "reduce_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
+    "scalar_mul", "reduce_segments", "multiexp_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
     "Codec", "FlbError", "library_path", "op_cost", "keygen_gpu", "miller_rabin", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
     "reduce_segments_host", "pack_encrypt_host_multi",
 ]
@@ -227,8 +227,28 @@ def reduce_segments(pub: PublicKey, c: torch.Tensor, offsets: torch.Tensor, idx:
     if out is None:
         out = torch.empty((S, pub.ct_words), dtype=torch.int32, device=c.device)
     _check_batch(out, pub.ct_words, "out")
-    check("flb_reduce_segments", LIB.flb_reduce_segments(pub.handle, _ptr(c), L, _ptr(idx), _ptr(offsets), S,
+    nent = idx.shape[0] if idx is not None else L
+    check("flb_reduce_segments", LIB.flb_reduce_segments(pub.handle, _ptr(c), L, _ptr(idx), nent, _ptr(offsets), S,
                                                          max_segment_len, _ptr(out), _stream(stream)))
+    return out
+
+
+def multiexp_segments(pub: PublicKey, c: torch.Tensor, e: torch.Tensor, offsets: torch.Tensor,
+                      idx: Optional[torch.Tensor] = None, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
+    """out[j] = prod_{t in seg j} c[idx[t]]^(e[t]) mod n^2 (per-entry exponents e [entries, e_words])."""
+    L = _check_batch(c, pub.ct_words, "c")
+    if offsets.dtype != torch.int64 or not offsets.is_cuda or offsets.dim() != 1 or not offsets.is_contiguous():
+        raise ValueError("offsets must be a contiguous CUDA int64 vector")
+    S = offsets.shape[0] - 1
+    nent = e.shape[0]
+    _check_batch(e, e.shape[1], "e")
+    if idx is not None and (idx.dtype != torch.int64 or not idx.is_cuda or not idx.is_contiguous()):
+        raise ValueError("idx must be a contiguous CUDA int64 vector")
+    if out is None:
+        out = torch.empty((S, pub.ct_words), dtype=torch.int32, device=c.device)
+    _check_batch(out, pub.ct_words, "out")
+    check("flb_multiexp_segments", LIB.flb_multiexp_segments(pub.handle, _ptr(c), L, _ptr(idx), _ptr(e), e.shape[1],
+                                                             _ptr(offsets), S, nent, _ptr(out), _stream(stream)))
     return out
 
 

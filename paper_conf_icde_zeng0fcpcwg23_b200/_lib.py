@@ -49,7 +49,8 @@ SIGNATURES = {
     "flb_decrypt": (ctypes.c_int, [_P, _P, _P, _SZ, _P]),
     "flb_add": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
     "flb_scalar_mul": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),
-    "flb_reduce_segments": (ctypes.c_int, [_P, _P, _SZ, _P, _P, _SZ, _SZ, _P, _P]),
+    "flb_reduce_segments": (ctypes.c_int, [_P, _P, _SZ, _P, _SZ, _P, _SZ, _SZ, _P, _P]),
+    "flb_multiexp_segments": (ctypes.c_int, [_P, _P, _SZ, _P, _P, _U32, _P, _SZ, _SZ, _P, _P]),
     "flb_pack": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _P]),
     "flb_unpack": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P, _P]),
     "flb_unpack_sums": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _P]),

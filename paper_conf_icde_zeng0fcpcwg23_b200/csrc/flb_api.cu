@@ -471,6 +471,25 @@ int run_modpow(const flb_pub* K, const uint32_t* dev, const uint32_t* sched, con
 }
 
 template <int X, int T>
+int run_horner(const flb_pub* K, const uint32_t* dev, const uint32_t* P, uint32_t planes, uint32_t* out, size_t nseg,
+               cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_horner<X, T>, nseg, &grid);
+  if (rc) return rc;
+  flb::HornerArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R1 = dev + K->o_R1;
+  A.R2 = dev + K->o_R2;
+  A.P = P;
+  A.K = planes;
+  A.out = out;
+  A.nseg = nseg;
+  flb::k_horner<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
 int run_mr(const uint32_t* cand, const uint32_t* bases, uint32_t rounds, uint64_t seed, uint64_t ctr0, uint32_t* verdict,
            size_t count, int bw, cudaStream_t st) {
   int grid;
@@ -543,10 +562,11 @@ int run_smul(const flb_pub* K, const uint32_t* dev, const uint32_t* c, const uin
 }
 
 template <int X, int T>
-int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t num_inputs, const int64_t* idx,
+int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t num_entries, const int64_t* idx,
                const int64_t* offsets, size_t nseg, size_t max_len, uint32_t* out, cudaStream_t st) {
   const int C = kReduceChunk;
-  if (max_len == 0) max_len = num_inputs;
+  const size_t num_inputs = num_entries;  // chunk bounds follow the entries (idx may repeat inputs)
+  if (max_len == 0 || max_len > num_entries) max_len = std::max<size_t>(num_entries, 1);
   int levels = 1;
   for (size_t cap = C; cap < max_len; cap *= C) levels++;
   // per-level buffers: chunk offsets [nseg+1], starts/ends [max_chunks], partials
@@ -846,15 +866,16 @@ int flb_scalar_mul(const flb_pub* K, const uint32_t* c, const uint32_t* e, uint3
 }
 
 int flb_reduce_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs, const int64_t* idx,
-                        const int64_t* offsets, size_t num_segments, size_t max_segment_len, uint32_t* out,
-                        void* stream) {
+                        size_t num_entries, const int64_t* offsets, size_t num_segments, size_t max_segment_len,
+                        uint32_t* out, void* stream) {
   if (!K || !offsets || !out) return fail(FLB_EINVAL, "null pointer");
-  if (num_inputs > 0 && !c) return fail(FLB_EINVAL, "null input");
+  if (num_entries > 0 && (!c || num_inputs == 0)) return fail(FLB_EINVAL, "null or empty input");
+  if (!idx && num_entries > num_inputs) return fail(FLB_EINVAL, "without idx, num_entries must be <= num_inputs");
   if (num_segments == 0) return FLB_OK;
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
-  FLB_DISPATCH_ENC(K->frame, run_reduce, K, dev, c, num_inputs, idx, offsets, num_segments, max_segment_len, out,
+  FLB_DISPATCH_ENC(K->frame, run_reduce, K, dev, c, num_entries, idx, offsets, num_segments, max_segment_len, out,
                    (cudaStream_t)stream);
 }
 
@@ -978,6 +999,90 @@ int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out
   } catch (const std::exception& ex) {
     return fail(FLB_EINVAL, ex.what());
   }
+}
+
+// Segmented multi-exponentiation (Hetero-LR's per-feature sum of residual x feature, C3):
+// Pippenger's bucket method on top of the segmented product kernel.
+int flb_multiexp_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs, const int64_t* idx, const uint32_t* e,
+                          uint32_t e_words, const int64_t* offsets, size_t num_segments, size_t num_entries, uint32_t* out,
+                          void* stream) {
+  if (!K || !offsets || !out || (num_entries && (!c || !e))) return fail(FLB_EINVAL, "null pointer");
+  if (e_words < 1 || e_words > 8) return fail(FLB_EINVAL, "e_words must be in [1, 8]");
+  if (num_segments == 0) return FLB_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint32_t s_words = K->s;
+  const uint64_t Kb = 32ull * e_words;
+  const uint64_t avg = num_entries / num_segments;
+  const char* force = getenv("FLB_MULTIEXP");
+  const bool naive = (force && std::string(force) == "naive") || avg < 256;
+  if (naive) {
+    // gather c[idx[t]] for every entry, scalar-mul by e_t, product per segment
+    Scratch rows, pw;
+    int rc = rows.alloc(std::max<size_t>(1, num_entries) * s_words * 4, st);
+    if (rc) return rc;
+    rc = pw.alloc(std::max<size_t>(1, num_entries) * s_words * 4, st);
+    if (rc) return rc;
+    if (num_entries) {
+      flb::k_gather_rows<<<grid_1d(num_entries * s_words), 256, 0, st>>>(c, idx, (int64_t)num_entries, s_words,
+                                                                          (uint32_t*)rows.p);
+      FLB_LAUNCH_CHECK();
+      rc = flb_scalar_mul(K, (const uint32_t*)rows.p, e, e_words, (uint32_t*)pw.p, num_entries, stream);
+      if (rc) return rc;
+    }
+    return flb_reduce_segments(K, (const uint32_t*)pw.p, num_entries, nullptr, num_entries, offsets, num_segments, 0,
+                               out, stream);
+  }
+  // window width minimising entries*W (bucket products) + W*cb*2^(cb-1) (bit planes), bucket count capped
+  uint32_t cb = 4;
+  double best = 1e300;
+  for (uint32_t t = 4; t <= 16; t++) {
+    const uint64_t W = (Kb + t - 1) / t;
+    if ((uint64_t)num_segments * W << t > (8ull << 20)) break;
+    const double cost = (double)num_entries * W + (double)num_segments * W * t * (double)(1ull << (t - 1));
+    if (cost < best) { best = cost; cb = t; }
+  }
+  const uint64_t W = (Kb + cb - 1) / cb;
+  const uint64_t nb = (uint64_t)num_segments * W << cb;
+  const uint64_t planes = W * cb, nplanes = (uint64_t)num_segments * planes, half = 1ull << (cb - 1);
+  Scratch s_cnt, s_off, s_sorted, s_B, s_idx2, s_off2, s_P;
+  int rc;
+  if ((rc = s_cnt.alloc((nb + 1) * 8, st)) || (rc = s_off.alloc((nb + 1) * 8, st)) ||
+      (rc = s_sorted.alloc(std::max<uint64_t>(1, num_entries * W) * 8, st)) || (rc = s_B.alloc(nb * s_words * 4, st)) ||
+      (rc = s_idx2.alloc(nplanes * half * 8, st)) || (rc = s_off2.alloc((nplanes + 1) * 8, st)) ||
+      (rc = s_P.alloc(nplanes * s_words * 4, st)))
+    return rc;
+  unsigned long long* cnt = (unsigned long long*)s_cnt.p;
+  int64_t* boff = (int64_t*)s_off.p;
+  FLB_CK(cudaMemsetAsync(cnt, 0, (nb + 1) * 8, st));
+  const int g = grid_1d(num_entries);
+  if (num_entries) {
+    flb::k_bucket<0><<<g, 256, 0, st>>>(offsets, (int64_t)num_segments, (int64_t)num_entries, idx, e, e_words,
+                                        (uint32_t)W, cb, cnt, nullptr);
+    FLB_LAUNCH_CHECK();
+  }
+  flb::k_scan_u64<<<1, 1024, 0, st>>>(cnt, (int64_t)nb, boff);
+  FLB_LAUNCH_CHECK();
+  FLB_CK(cudaMemcpyAsync(cnt, boff, nb * 8, cudaMemcpyDeviceToDevice, st));  // cursors = bucket starts
+  if (num_entries) {
+    flb::k_bucket<1><<<g, 256, 0, st>>>(offsets, (int64_t)num_segments, (int64_t)num_entries, idx, e, e_words,
+                                        (uint32_t)W, cb, cnt, (int64_t*)s_sorted.p);
+    FLB_LAUNCH_CHECK();
+  }
+  // bucket products, then bit-plane products, then Horner over the planes
+  rc = flb_reduce_segments(K, c, num_inputs, (const int64_t*)s_sorted.p, std::max<uint64_t>(1, num_entries * W), boff,
+                           nb, 0, (uint32_t*)s_B.p, stream);
+  if (rc) return rc;
+  flb::k_bitplane_index<<<grid_1d(nplanes * half), 256, 0, st>>>((int64_t)nplanes, cb, (int64_t*)s_idx2.p);
+  FLB_LAUNCH_CHECK();
+  flb::k_arange_offsets<<<grid_1d(nplanes + 1), 256, 0, st>>>((int64_t)nplanes, (int64_t)half, (int64_t*)s_off2.p);
+  FLB_LAUNCH_CHECK();
+  rc = flb_reduce_segments(K, (const uint32_t*)s_B.p, nb, (const int64_t*)s_idx2.p, nplanes * half,
+                           (const int64_t*)s_off2.p, nplanes, half, (uint32_t*)s_P.p, stream);
+  if (rc) return rc;
+  uint32_t* dev;
+  rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  FLB_DISPATCH_ENC(K->frame, run_horner, K, dev, (const uint32_t*)s_P.p, (uint32_t)planes, out, num_segments, st);
 }
 
 static int frame_key(uint32_t words, uint32_t* key) {

@@ -321,7 +321,8 @@ int flb_reduce_segments_host(const flb_pub* pub, const uint32_t* c_host, size_t 
   PCK(cudaMemcpyAsync(C->d_aux[0].p, aux, (num_segments + 1 + nidx) * 8, cudaMemcpyHostToDevice, st));
   const int64_t* d_off = (const int64_t*)C->d_aux[0].p;
   const int64_t* d_idx = idx_host ? d_off + num_segments + 1 : nullptr;
-  int rc = flb_reduce_segments(pub, (const uint32_t*)C->d_in[0].p, num_inputs, d_idx, d_off, num_segments,
+  const size_t nent = idx_host ? nidx : (size_t)offsets_host[num_segments];
+  int rc = flb_reduce_segments(pub, (const uint32_t*)C->d_in[0].p, num_inputs, d_idx, nent, d_off, num_segments,
                                max_segment_len, (uint32_t*)C->d_out[0].p, st);
   if (rc) return lib_err(rc, "flb_reduce_segments");
   PCK(cudaMemcpyAsync(C->pin_out[0].p, C->d_out[0].p, num_segments * ctw * 4, cudaMemcpyDeviceToHost, st));

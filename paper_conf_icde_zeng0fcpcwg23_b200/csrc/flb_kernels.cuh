@@ -572,6 +572,153 @@ __global__ void k_sieve(const uint32_t* __restrict__ cand, uint64_t count, uint3
   }
 }
 
+// ----------------------------------------------------------------------------- multi-exponentiation
+// Pippenger bucket method for out_j = prod_{t in seg j} c[idx t]^(e_t): the exponent bits are
+// cut into W windows of cb bits; bucket (j, w, v) collects the inputs whose window-w digit is v.
+
+// segment of entry t (offsets non-decreasing, nseg >= 1)
+__device__ __forceinline__ int64_t seg_of(const int64_t* __restrict__ off, int64_t nseg, int64_t t) {
+  int64_t lo = 0, hi = nseg - 1;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) >> 1;
+    if (off[mid] <= t) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ uint32_t exp_digit(const uint32_t* __restrict__ e, uint32_t e_words, uint32_t lo, uint32_t cb) {
+  const uint32_t word = lo >> 5, off = lo & 31u;
+  uint64_t v = (word < e_words) ? __ldg(e + word) : 0u;
+  if (word + 1 < e_words) v |= (uint64_t)__ldg(e + word + 1) << 32;
+  return (uint32_t)(v >> off) & ((1u << cb) - 1u);
+}
+
+// pass 0: count bucket sizes; pass 1: scatter input indices into buckets (cursor = bucket starts)
+template <int PASS>
+__global__ void k_bucket(const int64_t* __restrict__ off, int64_t nseg, int64_t nent, const int64_t* __restrict__ idx,
+                         const uint32_t* __restrict__ e, uint32_t e_words, uint32_t W, uint32_t cb,
+                         unsigned long long* __restrict__ cnt_or_cursor, int64_t* __restrict__ sorted) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nent; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = seg_of(off, nseg, t);
+    const uint32_t* et = e + t * e_words;
+    for (uint32_t w = 0; w < W; w++) {
+      const uint32_t v = exp_digit(et, e_words, w * cb, cb);
+      if (!v) continue;
+      const uint64_t b = ((uint64_t)j * W + w) << cb | v;
+      if (PASS == 0) {
+        atomicAdd(cnt_or_cursor + b, 1ull);
+      } else {
+        const unsigned long long pos = atomicAdd(cnt_or_cursor + b, 1ull);
+        sorted[pos] = idx ? idx[t] : t;
+      }
+    }
+  }
+}
+
+// exclusive scan of n counters (one block): out[i] = sum_{k<i} in[k], out[n] = total
+__global__ void k_scan_u64(const unsigned long long* __restrict__ in, int64_t n, int64_t* __restrict__ out) {
+  __shared__ long long warp_sums[32];
+  __shared__ long long carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int64_t base = 0; base < n; base += blockDim.x) {
+    const int64_t i = base + threadIdx.x;
+    const long long v = i < n ? (long long)in[i] : 0;
+    long long x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) warp_sums[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      long long s = (lane < (int)(blockDim.x >> 5)) ? warp_sums[lane] : 0;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const long long y = __shfl_up_sync(FULL, s, o);
+        if (lane >= o) s += y;
+      }
+      warp_sums[lane] = s;
+    }
+    __syncthreads();
+    const long long before = carry + (wid ? warp_sums[wid - 1] : 0) + x - v;
+    if (i < n) out[i] = before;
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) carry = before + v;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) out[n] = carry;
+}
+
+// bit-plane index: for plane p = (j, w, bit) list the buckets (j, w, v) with that bit of v set
+__global__ void k_bitplane_index(int64_t nplanes, uint32_t cb, int64_t* __restrict__ idx2) {
+  const int64_t half = (int64_t)1 << (cb - 1);
+  const int64_t total = nplanes * half;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = t / half, r = t - p * half;
+    const uint32_t bit = (uint32_t)(p % cb);
+    const int64_t jw = p / cb;
+    // r-th value v in [1, 2^cb) with bit `bit` set: insert a 1 at position `bit` into r
+    const uint64_t low = (uint64_t)r & ((1ull << bit) - 1), high = ((uint64_t)r >> bit) << (bit + 1);
+    const uint64_t v = high | (1ull << bit) | low;
+    idx2[t] = (jw << cb) | (int64_t)v;
+  }
+}
+
+__global__ void k_arange_offsets(int64_t n, int64_t step, int64_t* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = i * step;
+}
+
+struct HornerArgs {
+  ModRef N2;
+  const uint32_t* R1;
+  const uint32_t* R2;
+  const uint32_t* P;   // [nseg][K][S] bit-plane products (plane k = w * cb + bit)
+  uint32_t K;
+  uint32_t* out;       // [nseg][S]
+  uint64_t nseg;
+};
+
+// out_j = prod_k P_{j,k}^(2^k) by Horner from the top bit (Montgomery domain inside).
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_horner(const HornerArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  uint32_t n[X];
+  load_mod<X, T>(n, A.N2);
+  const uint32_t n0inv = A.N2.n0inv;
+  for (uint64_t base = g.wg0; base < A.nseg; base += g.G) {
+    const uint64_t j = base + (g.gid - g.wg0);
+    const bool valid = j < A.nseg;
+    uint32_t acc[X], b[X], r2[X];
+    load_const<X, T>(acc, A.R1);
+    load_const<X, T>(r2, A.R2);
+#pragma unroll 1
+    for (int k = (int)A.K - 1; k >= 0; k--) {
+      mont_sqr<X, T>(acc, acc, n, n0inv);
+      load_elem<X, T>(b, A.P + (j * A.K + (uint64_t)k) * S, S, valid);
+      mont_mul<X, T>(b, b, r2, n, n0inv);
+      mont_mul<X, T>(acc, acc, b, n, n0inv);
+    }
+    set_one<X, T>(b);
+    mont_mul<X, T>(acc, acc, b, n, n0inv);
+    if (valid) store_limbs<X>(A.out + j * S + g.k * X, acc);
+  }
+}
+
+// rows[i] = c[idx[i]] (gather, one thread per word)
+__global__ void k_gather_rows(const uint32_t* __restrict__ c, const int64_t* __restrict__ idx, int64_t n, uint32_t S,
+                              uint32_t* __restrict__ out) {
+  const int64_t total = n * S;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = t / S;
+    out[t] = c[(idx ? idx[i] : i) * S + (t - i * S)];
+  }
+}
+
 // ----------------------------------------------------------------------------- hom-add
 struct AddArgs {
   ModRef N2;

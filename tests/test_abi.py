@@ -101,8 +101,9 @@ def test_batch_calls_validate_before_launch():
     assert L.flb_decrypt(priv.handle, None, None, 4, None) == -1
     assert L.flb_add(pub.handle, None, None, None, 4, None) == -1
     assert L.flb_scalar_mul(pub.handle, 16, 16, 0, 16, 4, None) == -1  # e_words = 0
-    assert L.flb_reduce_segments(pub.handle, None, 3, None, None, 2, 0, None, None) == -1
+    assert L.flb_reduce_segments(pub.handle, None, 3, None, 3, None, 2, 0, None, None) == -1
     assert "null" in L.flb_last_error().decode()
+    assert L.flb_reduce_segments(pub.handle, 16, 3, None, 4, 16, 2, 0, 16, None) == -1  # entries > inputs, no idx
     # count = 0 is a no-op that needs no device
     assert L.flb_encrypt(pub.handle, 16, None, 0, 0, 16, 0, None) == 0
     bad = [(1.0, 29, 3, 32, 32), (1.0, 29, 4, 33, 1), (0.0, 29, 3, 32, 1), (1.0, 53, 11, 64, 1), (1.0, 29, 3, 32, 0)]
