@@ -123,6 +123,14 @@ struct flb_priv {
   } pr[2];
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
   size_t o_q2invR = 0, o_enc_sched = 0;  // key-holder encryption: (q^2)^-1 R mod p^2, schedule of n
+  // key-holder encryption v2 (r^n mod P^2 = (r^Q mod P)^P mod P^2): half-frame moduli and schedules
+  uint32_t H = 0;                         // half-frame limbs (0: v2 not used for this key size)
+  struct Half {
+    uint32_t n0inv;
+    size_t o_P, o_R2, o_R3;
+  } half[2];
+  H::Schedule sched_p, sched_q;           // exponents p and q
+  size_t o_sched_p = 0, o_sched_q = 0;
   uint32_t n_n0inv = 0;
   Blob blob;
   DevBlob dev;
@@ -230,6 +238,28 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
     const Limbs q2inv = Cp2.pow(H::mod(V->pr[1].P2, V->pr[0].P2), e);
     V->o_q2invR = V->blob.put(Cp2.to(q2inv), sp);
     V->o_enc_sched = V->blob.put_raw(V->pub->enc.ops);
+  }
+  {
+    // v2 half frame: the smallest supported frame holding p; used only when it is below sp
+    uint32_t Hf = 0;
+    const uint32_t pw = (uint32_t)((H::bits(V->p) + 31) / 32);
+    for (uint32_t f : {32u, 64u, 96u, 128u})
+      if (pw <= f) { Hf = f; break; }
+    if (Hf && Hf < sp) {
+      V->H = Hf;
+      for (int i = 0; i < 2; i++) {
+        const Limbs P = H::resized(i == 0 ? V->p : V->q, Hf);
+        H::MontCtx C(P);
+        V->half[i].n0inv = C.n0inv;
+        V->half[i].o_P = V->blob.put(P, Hf);
+        V->half[i].o_R2 = V->blob.put(C.R2, Hf);
+        V->half[i].o_R3 = V->blob.put(H::mont(C.R2, C.R2, P, C.n0inv), Hf);
+      }
+      V->sched_p = H::best_schedule(V->p, 7);
+      V->sched_q = H::best_schedule(V->q, 7);
+      V->o_sched_p = V->blob.put_raw(V->sched_p.ops);
+      V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
+    }
   }
   // CRT recombination constants
   H::MontCtx Cn(V->pub->n), Cp(V->p);
@@ -514,6 +544,74 @@ int run_mr(const uint32_t* cand, const uint32_t* bases, uint32_t rounds, uint64_
   return FLB_OK;
 }
 
+template <int X, int T>
+int run_crt_pre(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* y,
+                size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_crt_pre<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->sched_p.table, V->sched_q.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->H * 4, st);
+  if (rc) return rc;
+  flb::CrtPreArgs A;
+  for (int i = 0; i < 2; i++) {
+    A.P[i] = {dev + V->half[i].o_P, V->half[i].n0inv};
+    A.R2[i] = dev + V->half[i].o_R2;
+    A.R3[i] = dev + V->half[i].o_R3;
+    const H::Schedule& sc_i = i == 0 ? V->sched_q : V->sched_p;  // exponent: the other prime
+    A.sched[i] = dev + (i == 0 ? V->o_sched_q : V->o_sched_p);
+    A.sched_len[i] = (int)sc_i.ops.size();
+    A.table[i] = sc_i.table;
+  }
+  A.nbits = V->pub->nbits;
+  A.pt_words = V->pub->sp;
+  A.r = r;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.y = y;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_crt_pre<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_encrypt_crt2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
+                     size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt_crt2<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->sched_p.table, V->sched_q.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->pub->sp * 4, st);
+  if (rc) return rc;
+  flb::EncCrt2Args A;
+  for (int i = 0; i < 2; i++) {
+    A.P2[i] = {dev + V->pr[i].o_P2, V->pr[i].P2_n0inv};
+    A.R2[i] = dev + V->pr[i].o_R2;
+    A.nR[i] = dev + V->pr[i].o_nR;
+    const H::Schedule& sc_i = i == 0 ? V->sched_p : V->sched_q;  // exponent P for P^2
+    A.sched[i] = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
+    A.sched_len[i] = (int)sc_i.ops.size();
+    A.table[i] = sc_i.table;
+  }
+  A.q2 = dev + V->pr[1].o_P2;
+  A.q2invR = dev + V->o_q2invR;
+  A.m = m;
+  A.y = y;
+  A.H = V->H;
+  A.c = c;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt_crt2<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
 template <int X, int T, bool DEBUG>
 int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
             cudaStream_t st) {
@@ -716,7 +814,19 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       *limb_products = mm * csp + lp;
       return FLB_OK;
     }
-    case 4: {  // key-holder encryption: per prime 1 + table + schedule + 2 at sp; CRT 1 + plain product
+    case 4: {  // key-holder encryption
+      if (!V) return fail(FLB_EINVAL, "key-holder cost needs the private key");
+      const char* v1 = getenv("FLB_CRT_V1");
+      if (V->H && !(v1 && atoi(v1) == 1)) {
+        // v2: per prime, stage 1 at the half frame (2 entry + table + schedule(Q) + exit) and stage 2
+        // at sp (entry + table + schedule(P) + m n + final); CRT 1 + plain product
+        const uint64_t h = V->H, ch = 2 * h * h + h;
+        const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
+        const uint64_t s2 = (1 + sched_mults(V->sched_p) + 2) + (1 + sched_mults(V->sched_q) + 2) + 1;
+        *mont_muls = s1 + s2;
+        *limb_products = s1 * ch + s2 * csp + sp * sp;
+        return FLB_OK;
+      }
       const uint64_t per = 1 + sched_mults(P->enc) + 2;
       *mont_muls = 2 * per + 1;
       *limb_products = (2 * per + 1) * csp + sp * sp;
@@ -825,6 +935,9 @@ int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count,
   FLB_DISPATCH_DEC(V->pub->frame, run_decrypt, V, dev, c, m, count, (cudaStream_t)stream);
 }
 
+static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                          uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st);
+
 int flb_encrypt_crt(const flb_priv* V, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0,
                     uint32_t* c, size_t count, void* stream) {
   if (!V || !m || !c) return fail(FLB_EINVAL, "null pointer");
@@ -832,6 +945,8 @@ int flb_encrypt_crt(const flb_priv* V, const uint32_t* m, const uint32_t* r, uin
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
   if (rc) return rc;
+  const char* v1 = getenv("FLB_CRT_V1");
+  if (V->H && !(v1 && atoi(v1) == 1)) return encrypt_crt_v2(V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
   FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt, V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 
@@ -1083,6 +1198,31 @@ int flb_multiexp_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs
   rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
   FLB_DISPATCH_ENC(K->frame, run_horner, K, dev, (const uint32_t*)s_P.p, (uint32_t)planes, out, num_segments, st);
+}
+
+static int frame_key(uint32_t words, uint32_t* key);
+
+static int crt_pre_dispatch(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0,
+                            uint32_t* y, size_t count, cudaStream_t st) {
+  uint32_t key;
+  int rc = frame_key(V->H, &key);
+  if (rc) return rc;
+  FLB_DISPATCH_ENC(key, run_crt_pre, V, dev, r, seed, ctr0, y, count, st);
+}
+
+static int crt2_dispatch(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
+                         size_t count, cudaStream_t st) {
+  FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt2, V, dev, m, y, c, count, st);
+}
+
+static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                          uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  Scratch ys;
+  int rc = ys.alloc((size_t)2 * count * V->H * 4, st);
+  if (rc) return rc;
+  rc = crt_pre_dispatch(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
+  if (rc) return rc;
+  return crt2_dispatch(V, dev, m, (const uint32_t*)ys.p, c, count, st);
 }
 
 static int frame_key(uint32_t words, uint32_t* key) {

@@ -69,12 +69,18 @@ __device__ __forceinline__ void set_one(uint32_t (&r)[X]) {
   if (k == 0) r[0] = 1;
 }
 
-// Load limbs [k*X, k*X+X) of an element with `words` limbs (words may be < X*T: the rest are 0).
+// Load limbs [k*X, k*X+X) of an element with `words` limbs (words may be < X*T: the rest are 0;
+// a chunk straddling `words` is read word by word so no lane reads past the element).
 template <int X, int T>
 __device__ __forceinline__ void load_elem(uint32_t (&r)[X], const uint32_t* base, uint32_t words, bool valid) {
   const int k = (int)(lane_id() & (T - 1));
-  if (valid && (uint32_t)(k * X) < words) load_limbs<X>(r, base + k * X);
-  else zero_limbs<X>(r);
+  const uint32_t w0 = (uint32_t)(k * X);
+  if (valid && w0 + X <= words) {
+    load_limbs<X>(r, base + w0);
+  } else {
+#pragma unroll
+    for (int j = 0; j < X; j++) r[j] = (valid && w0 + j < words) ? __ldg(base + w0 + j) : 0u;
+  }
 }
 
 // ----------------------------------------------------------------------------- Philox4x32-10
@@ -93,12 +99,12 @@ __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 key) {
 // r for element `index`: pt_words Philox words, bits >= nbits-1 cleared, 0 -> 1.
 template <int X, int T>
 __device__ __forceinline__ void philox_r(uint32_t (&r)[X], uint64_t seed, uint64_t index, uint32_t pt_words,
-                                         uint32_t nbits) {
+                                         uint32_t nbits, uint32_t woff = 0, bool fix_zero = true) {
   const int k = (int)(lane_id() & (T - 1));
   const uint2 key = make_uint2((uint32_t)seed, (uint32_t)(seed >> 32));
 #pragma unroll
   for (int v = 0; v < X / 4; v++) {
-    const uint32_t w0 = (uint32_t)(k * X + 4 * v);
+    const uint32_t w0 = woff + (uint32_t)(k * X + 4 * v);
     uint4 o = make_uint4(0, 0, 0, 0);
     if (w0 < pt_words) o = philox4x32_10(make_uint4((uint32_t)index, (uint32_t)(index >> 32), w0 / 4, 0), key);
     r[4 * v] = o.x; r[4 * v + 1] = o.y; r[4 * v + 2] = o.z; r[4 * v + 3] = o.w;
@@ -106,15 +112,17 @@ __device__ __forceinline__ void philox_r(uint32_t (&r)[X], uint64_t seed, uint64
   const uint32_t lim = nbits - 1;  // keep bits [0, nbits-1)
 #pragma unroll
   for (int j = 0; j < X; j++) {
-    const uint32_t w = (uint32_t)(k * X + j);
+    const uint32_t w = woff + (uint32_t)(k * X + j);
     if (w >= pt_words || 32u * w >= lim) r[j] = 0;
     else if (32u * (w + 1) > lim) r[j] &= (1u << (lim - 32u * w)) - 1u;
   }
-  const bool nz = !all_zero<X>(r);
-  const uint32_t bal = __ballot_sync(FULL, nz);
-  const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
-  const uint32_t gm = (T == 32) ? 0xffffffffu : (((1u << T) - 1u) << base);
-  if ((bal & gm) == 0 && k == 0) r[0] = 1;
+  if (fix_zero) {
+    const bool nz = !all_zero<X>(r);
+    const uint32_t bal = __ballot_sync(FULL, nz);
+    const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
+    const uint32_t gm = (T == 32) ? 0xffffffffu : (((1u << T) - 1u) << base);
+    if ((bal & gm) == 0 && k == 0) r[0] = 1;
+  }
 }
 
 // ----------------------------------------------------------------------------- modexp
@@ -716,6 +724,135 @@ __global__ void k_gather_rows(const uint32_t* __restrict__ c, const int64_t* __r
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i = t / S;
     out[t] = c[(idx ? idx[i] : i) * S + (t - i * S)];
+  }
+}
+
+// ----------------------------------------------------------------------------- key-holder encrypt, v2
+// r^n mod P^2 = ((r^Q mod P))^P mod P^2 for {P, Q} = {p, q}: x^P mod P^2 depends only on x mod P
+// ((y + kP)^P = y^P mod P^2 by the binomial theorem), and r^n = (r^Q)^P.  Stage 1 (this kernel,
+// half-size frame): y_P = r^Q mod P.  Stage 2 (k_encrypt_crt2, P^2 frame): c_P = (1 + mn) y_P^P
+// mod P^2, then the CRT combine of k_encrypt_crt.  Exact for every r (r = 0 mod P gives 0 both ways).
+struct CrtPreArgs {
+  ModRef P[2];             // p, q in the half frame
+  const uint32_t* R2[2];   // R^2 mod P (half frame)
+  const uint32_t* R3[2];   // R^3 mod P
+  const uint32_t* sched[2];  // exponent Q (the other prime) for P
+  int sched_len[2], table[2];
+  uint32_t nbits;          // bits(n)
+  uint32_t pt_words;       // sp (the frame of r)
+  const uint32_t* r;       // [count][pt_words] or null (Philox)
+  uint64_t seed, ctr0;
+  uint32_t* y;             // [2][count][H]
+  uint64_t count;
+  uint32_t* scratch;
+};
+
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_DEC) k_crt_pre(const CrtPreArgs A) {
+  constexpr int H = X * T;
+  const Grid<T> g;
+  uint32_t* tab = A.scratch + (size_t)g.gid * H;
+  const size_t stride = (size_t)g.G * H;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+#pragma unroll 1
+    for (int P = 0; P < 2; P++) {
+      uint32_t n[X], lo[X], hi[X], b[X], x[X];
+      load_mod<X, T>(n, A.P[P]);
+      const uint32_t n0inv = A.P[P].n0inv;
+      if (A.r) {
+        load_elem<X, T>(lo, A.r + e * A.pt_words, min(A.pt_words, (uint32_t)H), valid);
+        if (A.pt_words > (uint32_t)H) load_elem<X, T>(hi, A.r + e * A.pt_words + H, A.pt_words - H, valid);
+        else zero_limbs<X>(hi);
+      } else {
+        // the same words philox_r draws for the whole r: low H words, then the rest; r = 0 -> 1
+        philox_r<X, T>(lo, A.seed, A.ctr0 + e, A.pt_words, A.nbits, 0, false);
+        philox_r<X, T>(hi, A.seed, A.ctr0 + e, A.pt_words, A.nbits, H, false);
+        const bool nz = !(all_zero<X>(lo) && all_zero<X>(hi));
+        const uint32_t bal = __ballot_sync(FULL, nz);
+        const int gb = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
+        const uint32_t gm = (T == 32) ? 0xffffffffu : (((1u << T) - 1u) << gb);
+        if ((bal & gm) == 0 && g.k == 0) lo[0] = 1;
+      }
+      load_const<X, T>(b, A.R2[P]);
+      mont_mul<X, T>(lo, lo, b, n, n0inv);                   // r_lo R mod P
+      load_const<X, T>(b, A.R3[P]);
+      mont_mul<X, T>(hi, hi, b, n, n0inv);                   // r_hi R^2 mod P
+      const uint32_t cy = grp_add<X, T>(x, lo, hi);
+      grp_cond_sub<X, T>(x, n, cy);                          // r R mod P
+      modexp_sched<X, T>(lo, x, A.sched[P], A.sched_len[P], A.table[P], tab, stride, n, n0inv);
+      set_one<X, T>(b);
+      mont_mul<X, T>(lo, lo, b, n, n0inv);                   // y_P = r^Q mod P
+      if (valid) store_limbs<X>(A.y + ((uint64_t)P * A.count + e) * H + g.k * X, lo);
+    }
+  }
+}
+
+struct EncCrt2Args {
+  ModRef P2[2];
+  const uint32_t* R2[2];   // R^2 mod P^2 (sp frame)
+  const uint32_t* nR[2];
+  const uint32_t* q2;
+  const uint32_t* q2invR;
+  const uint32_t* sched[2];  // exponent P for P^2
+  int sched_len[2], table[2];
+  const uint32_t* m;       // [count][sp]
+  const uint32_t* y;       // [2][count][H]
+  uint32_t H;
+  uint32_t* c;             // [count][2 sp]
+  uint64_t count;
+  uint32_t* scratch;
+};
+
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_DEC) k_encrypt_crt2(const EncCrt2Args A) {
+  constexpr int S = X * T;  // sp
+  const Grid<T> g;
+  uint32_t* tab = A.scratch + (size_t)g.gid * S;
+  const size_t stride = (size_t)g.G * S;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t cres[2][X];
+#pragma unroll 1
+    for (int P = 0; P < 2; P++) {
+      uint32_t n[X], x[X], b[X], acc[X];
+      load_mod<X, T>(n, A.P2[P]);
+      const uint32_t n0inv = A.P2[P].n0inv;
+      load_elem<X, T>(x, A.y + ((uint64_t)P * A.count + e) * A.H, A.H, valid);
+      load_const<X, T>(b, A.R2[P]);
+      mont_mul<X, T>(x, x, b, n, n0inv);                       // y R mod P^2
+      modexp_sched<X, T>(acc, x, A.sched[P], A.sched_len[P], A.table[P], tab, stride, n, n0inv);  // y^P R
+      load_elem<X, T>(x, A.m + e * S, S, valid);
+      load_const<X, T>(b, A.nR[P]);
+      mont_mul<X, T>(x, x, b, n, n0inv);                       // m n mod P^2
+      set_one<X, T>(b);
+      const uint32_t cy = grp_add<X, T>(x, x, b);
+      grp_cond_sub<X, T>(x, n, cy);                            // 1 + m n mod P^2
+      mont_mul<X, T>(acc, acc, x, n, n0inv);                   // c_P = (1 + mn) r^n mod P^2
+#pragma unroll
+      for (int j = 0; j < X; j++) {
+        if (P == 0) cres[0][j] = acc[j];
+        else cres[1][j] = acc[j];
+      }
+    }
+    uint32_t n[X], d[X], t[X], hi[X];
+    load_mod<X, T>(n, A.P2[0]);
+    const uint32_t br = grp_sub<X, T>(d, cres[0], cres[1]);
+#pragma unroll
+    for (int j = 0; j < X; j++) t[j] = br ? n[j] : 0u;
+    grp_add<X, T>(d, d, t);
+    load_const<X, T>(t, A.q2invR);
+    mont_mul<X, T>(d, d, t, n, A.P2[0].n0inv);
+    load_const<X, T>(t, A.q2);
+    mul_full<X, T>(d, hi, d, t);
+    const uint32_t cy = grp_add<X, T>(d, d, cres[1]);
+    grp_add_small<X, T>(hi, cy);
+    if (valid) {
+      store_limbs<X>(A.c + e * (2 * S) + g.k * X, d);
+      store_limbs<X>(A.c + e * (2 * S) + S + g.k * X, hi);
+    }
   }
 }
 
