@@ -371,7 +371,8 @@ def run_flb(args):
     # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
     if args.encrypt == "keyholder":
         enc_mm, enc_lp = flb.op_cost(priv, "encrypt_crt")
-        enc_kernel = "k_encrypt_crt<16,4>"
+        enc_kernel = ("k_encrypt_crt<16,4>" if os.environ.get("FLB_CRT_V1") == "1"
+                      else "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)")
     else:
         enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
         enc_kernel = "k_encrypt<16,8>"
