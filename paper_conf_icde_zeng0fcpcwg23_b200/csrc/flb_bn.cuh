@@ -303,8 +303,15 @@ template <int X, int T>
 __device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
                                                 uint32_t n0inv);
 
+template <int X, int T>
+__device__ __forceinline__ void mont_sqr_split(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
+                                               uint32_t n0inv);
+
 #ifndef FLB_SQR_BLOCKS
 #define FLB_SQR_BLOCKS 0  // measured slower on B200; kept as a parity-tested experiment
+#endif
+#ifndef FLB_SQR_SPLIT
+#define FLB_SQR_SPLIT 0  // bit-exact but measured slower on B200; parity-tested experiment
 #endif
 
 template <int X, int T>
@@ -312,6 +319,8 @@ __device__ __forceinline__ void mont_sqr(uint32_t (&r)[X], const uint32_t (&a)[X
                                          uint32_t n0inv) {
   if constexpr (FLB_SQR_BLOCKS && T >= 4) {
     mont_sqr_blocks<X, T>(r, a, n, n0inv);
+  } else if constexpr (FLB_SQR_SPLIT && T >= 2 && X >= 8 && X % 8 == 0) {
+    mont_sqr_split<X, T>(r, a, n, n0inv);
   } else {
     stage<X, T>(a);
     mont_mul_staged<X, T>(r, a, n, n0inv);
@@ -554,6 +563,156 @@ __device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t
   const uint32_t over1 = collapse<X, T>(r, E, O, pend);
   const uint32_t over2 = grp_add<X, T>(r, r, th);
   grp_cond_sub<X, T>(r, n, over1 | over2);
+}
+
+// ----------------------------------------------------------------------------- split squaring
+// Montgomery squaring with a quarter of the square's limb products moved out of the reduced part.
+// With B = 2^(32 S/2), R = B^2 and a = L + H B (L, H the low / high halves of a):
+//   a^2 = t_A + H^2 R,   t_A = L^2 + 2 L H B = L (L + 2 H B),
+// so a^2 R^-1 = (t_A + m N) / R + H^2 (mod N) for the m that REDC(t_A) picks: H^2 R is an exact
+// multiple of R and needs no reduction.  The reduced part is a CIOS over the S/2 multiplier words of
+// L against a'' = L + 2 H B (phase 1, S/2 full steps) followed by S/2 reduce-only steps (phase 2);
+// the plain half-size square H^2 is spread over all T lanes (X/2 words each) and its rows are
+// interleaved with phase 2, whose m-broadcast latency they hide.  Limb products: S^2/2 + S^2 + S^2/4
+// = 1.75 S^2 instead of CIOS's 2 S^2.  Bound: (t_A + m N)/R + H^2 = (a^2 + m N)/R < 2N for a < N, so
+// one conditional subtraction canonicalises, as for mont_mul.
+//
+// Phase-1 step: cios_step<REDUCE> plus `top` added at word X of the lane (word S of the group for
+// lane T-1: the product of b_i with the 2H top bit).
+template <int X, int T>
+__device__ __forceinline__ void cios_step_top(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
+                                              const uint32_t (&a)[X], uint32_t bi, uint32_t top,
+                                              const uint32_t (&n)[X], uint32_t n0inv) {
+  const int k = (int)(lane_id() & (T - 1));
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
+  chain_odd<X, true>(O, a, bi);
+  chain_even<X>(E, a, bi);
+  const uint32_t m = __shfl_sync(FULL, E[0], 0, T) * n0inv;
+  chain_even<X>(E, n, m);
+  chain_odd<X, false>(O, n, m);
+  // after both chains (their closing addc into E[X] / O[X] assume small top words); the shift
+  // below moves E[X] into a regular chain word, so a large value there is safe
+  asm volatile("add.cc.u32 %0, %0, %2;\n\taddc.u32 %1, %1, 0;" : "+r"(E[X]), "+r"(O[X]) : "r"(top));
+  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
+  if (k == T - 1) up = 0;
+  pend = E[1];
+  uint32_t nE[X + 1], nO[X + 1];
+#pragma unroll
+  for (int t = 0; t <= X; t++) nE[t] = O[t];
+#pragma unroll
+  for (int t = 0; t + 2 <= X; t++) nO[t] = E[t + 2];
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[X - 2]) : "r"(up));
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[X - 1]));
+  nO[X] = 0;
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
+}
+
+// Plain product row over HX words per lane (no reduction): acc += a * bi, shift one word down the
+// group.  Returns lane 0's word shifted out (the product's next low word; meaningful in lane 0).
+template <int HX, int T>
+__device__ __forceinline__ uint32_t prod_step(uint32_t (&E)[HX + 1], uint32_t (&O)[HX + 1], uint32_t& pend,
+                                              const uint32_t (&a)[HX], uint32_t bi) {
+  const int k = (int)(lane_id() & (T - 1));
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
+  chain_odd<HX, true>(O, a, bi);
+  chain_even<HX>(E, a, bi);
+  const uint32_t out = E[0];
+  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
+  if (k == T - 1) up = 0;
+  pend = E[1];
+  uint32_t nE[HX + 1], nO[HX + 1];
+#pragma unroll
+  for (int t = 0; t <= HX; t++) nE[t] = O[t];
+#pragma unroll
+  for (int t = 0; t + 2 <= HX; t++) nO[t] = E[t + 2];
+  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[HX - 2]) : "r"(up));
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[HX - 1]));
+  nO[HX] = 0;
+#pragma unroll
+  for (int t = 0; t <= HX; t++) { E[t] = nE[t]; O[t] = nO[t]; }
+  return out;
+}
+
+template <int X, int T>
+__device__ __forceinline__ void mont_sqr_split(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
+                                               uint32_t n0inv) {
+  constexpr int LD = X + 4, HX = X / 2, T2 = T / 2;
+  const int k = (int)(lane_id() & (T - 1));
+  stage<X, T>(a);
+  uint32_t* bs = stage_group<X, T>();
+  // a'' = L + 2 H B: lanes >= T/2 hold 2H (bits shifted up across lanes, none into lane T/2);
+  // the top bit of 2H is added as b_i * tb at word S (lane T-1, word X) in every phase-1 step
+  uint32_t ad[X];
+  {
+    uint32_t cin = __shfl_up_sync(FULL, a[X - 1], 1, T) >> 31;
+    if (k == T2) cin = 0;
+    const bool upper = k >= T2;
+#pragma unroll
+    for (int j = X - 1; j >= 1; j--) ad[j] = upper ? __funnelshift_l(a[j - 1], a[j], 1) : a[j];
+    ad[0] = upper ? ((a[0] << 1) | cin) : a[0];
+  }
+  const uint32_t tb = __shfl_sync(FULL, a[X - 1], T - 1, T) >> 31;
+  const uint32_t tmask = (tb != 0 && k == T - 1) ? 0xffffffffu : 0u;
+  uint32_t E[X + 1], O[X + 1], pend = 0;
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
+  // phase 1: multiplier words L_0 .. L_{S/2-1}
+#pragma unroll 1
+  for (int kk = 0; kk < T2; kk++) {
+    const uint32_t* row = bs + kk * LD;
+#pragma unroll
+    for (int jj = 0; jj < X; jj++) {
+      const uint32_t bi = row[jj];
+      cios_step_top<X, T>(E, O, pend, ad, bi, bi & tmask, n, n0inv);
+    }
+  }
+  // H spread over all T lanes: lane k holds H words [k HX, (k+1) HX) = staged row T/2 + k/2
+  uint32_t hl[HX];
+  {
+    const uint4* q = reinterpret_cast<const uint4*>(bs + (T2 + (k >> 1)) * LD + (k & 1) * HX);
+#pragma unroll
+    for (int v = 0; v < HX / 4; v++) {
+      const uint4 u = q[v];
+      hl[4 * v] = u.x; hl[4 * v + 1] = u.y; hl[4 * v + 2] = u.z; hl[4 * v + 3] = u.w;
+    }
+  }
+  __syncwarp();  // the L rows are dead from here on: phase 2 writes H^2's low words there
+  uint32_t E2[HX + 1], O2[HX + 1], pend2 = 0;
+#pragma unroll
+  for (int t = 0; t <= HX; t++) { E2[t] = 0; O2[t] = 0; }
+  // phase 2: reduce-only steps, each with one row of H^2 (multiplier word H_j = staged word S/2 + j)
+#pragma unroll 1
+  for (int kk = T2; kk < T; kk++) {
+    const uint32_t* row = bs + kk * LD;
+    uint32_t* outrow = bs + (kk - T2) * LD;
+#pragma unroll
+    for (int jj = 0; jj < X; jj++) {
+      const uint32_t hj = row[jj];
+      redc_step<X, T>(E, O, pend, n, n0inv);
+      const uint32_t w = prod_step<HX, T>(E2, O2, pend2, hl, hj);
+      if (k == 0) outrow[jj] = w;  // H^2 word (kk - T/2) X + jj
+    }
+  }
+  uint32_t over = collapse<X, T>(r, E, O, pend);
+  uint32_t h2[X];
+  {
+    uint32_t hh[HX];
+    collapse<HX, T>(hh, E2, O2, pend2);  // H^2 words S/2 + k HX ..; H^2 < R, no overflow
+    __syncwarp();                         // every lane has read its last H row
+    uint4* q = reinterpret_cast<uint4*>(bs + (T2 + (k >> 1)) * LD + (k & 1) * HX);
+#pragma unroll
+    for (int v = 0; v < HX / 4; v++) q[v] = make_uint4(hh[4 * v], hh[4 * v + 1], hh[4 * v + 2], hh[4 * v + 3]);
+    __syncwarp();
+    const uint4* p = reinterpret_cast<const uint4*>(bs + k * LD);
+#pragma unroll
+    for (int v = 0; v < X / 4; v++) {
+      const uint4 u = p[v];
+      h2[4 * v] = u.x; h2[4 * v + 1] = u.y; h2[4 * v + 2] = u.z; h2[4 * v + 3] = u.w;
+    }
+  }
+  over |= grp_add<X, T>(r, r, h2);
+  grp_cond_sub<X, T>(r, n, over);
 }
 
 // ----------------------------------------------------------------------------- loads / stores

@@ -1,0 +1,656 @@
+// flb_core.cuh — host-side runtime shared by the C ABI (flb_api.cu) and the per-frame kernel
+// instantiation units (flb_inst.cu): key structs, error state, launch configuration and the
+// run_* launchers.  Every run_<op><X, T> is explicitly instantiated in exactly one flb_inst.cu
+// object (one object per (X, T) frame split, compiled in parallel); flb_api.cu sees only the
+// extern declarations at the bottom of this file.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/flb_paillier.h"
+#include "flb_kernels.cuh"
+#include "host_bn.hpp"
+
+using flb::host::Limbs;
+namespace H = flb::host;
+
+namespace flb_rt {
+
+inline thread_local std::string g_err;
+
+inline int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+#define FLB_CK(call)                                                                    \
+  do {                                                                                  \
+    cudaError_t e_ = (call);                                                            \
+    if (e_ != cudaSuccess) return fail(FLB_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+constexpr int kBlock = 32;  // one warp per block: occupancy follows the register count exactly
+constexpr int kReduceChunk = 64;  // inputs per group in one reduction level
+
+// ----------------------------------------------------------------------------- constant blobs
+// All device constants of a key live in one buffer; Blob records word offsets.
+struct Blob {
+  std::vector<uint32_t> words;
+  size_t put(const Limbs& v, size_t w) {
+    // 16-byte align every array (uint4 loads)
+    while (words.size() % 4) words.push_back(0);
+    const size_t off = words.size();
+    Limbs r = H::resized(v, w);
+    words.insert(words.end(), r.begin(), r.end());
+    return off;
+  }
+  size_t put_raw(const std::vector<uint32_t>& v) {
+    while (words.size() % 4) words.push_back(0);
+    const size_t off = words.size();
+    words.insert(words.end(), v.begin(), v.end());
+    return off;
+  }
+};
+
+struct DevBlob {
+  std::mutex mu;
+  std::map<int, uint32_t*> per_dev;
+  ~DevBlob() {
+    for (auto& kv : per_dev) {
+      int cur;
+      if (cudaGetDevice(&cur) == cudaSuccess) {
+        cudaSetDevice(kv.first);
+        cudaFree(kv.second);
+        cudaSetDevice(cur);
+      }
+    }
+  }
+  // device copy of `b` on the current device (uploaded once)
+  int get(const Blob& b, uint32_t** out) {
+    int dev;
+    FLB_CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = per_dev.find(dev);
+    if (it != per_dev.end()) { *out = it->second; return FLB_OK; }
+    uint32_t* p = nullptr;
+    FLB_CK(cudaMalloc(&p, b.words.size() * 4));
+    FLB_CK(cudaMemcpy(p, b.words.data(), b.words.size() * 4, cudaMemcpyHostToDevice));
+    per_dev[dev] = p;
+    *out = p;
+    return FLB_OK;
+  }
+};
+
+inline int frame_for_bits(size_t nbits) {
+  if (nbits <= 1024) return 1024;
+  if (nbits <= 2048) return 2048;
+  if (nbits <= 3072) return 3072;
+  if (nbits <= 4096) return 4096;
+  return 0;
+}
+
+}  // namespace flb_rt
+
+using namespace flb_rt;
+
+// ----------------------------------------------------------------------------- key structs
+struct flb_pub {
+  uint32_t nbits = 0, frame = 0, s = 0, sp = 0;
+  Limbs n, n2;
+  uint32_t n2_n0inv = 0;
+  H::Schedule enc;
+  Blob blob;
+  size_t o_n2 = 0, o_R2 = 0, o_R1 = 0, o_nR = 0, o_RL = 0, o_sched = 0;
+  DevBlob dev;
+};
+
+struct flb_priv {
+  flb_pub* pub = nullptr;  // owned copy of the public half (for n / frame)
+  Limbs p, q;
+  struct Prime {
+    Limbs P, P2;
+    uint32_t P_n0inv, P2_n0inv;
+    H::Schedule sched;
+    size_t o_P, o_P2, o_R2, o_R3, o_Pinv, o_hR, o_sched;
+    size_t o_nR;  // n R mod P^2 (key-holder encryption)
+  } pr[2];
+  size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
+  size_t o_q2invR = 0, o_enc_sched = 0;  // key-holder encryption: (q^2)^-1 R mod p^2, schedule of n
+  // key-holder encryption v2 (r^n mod P^2 = (r^Q mod P)^P mod P^2): half-frame moduli and schedules
+  uint32_t H = 0;                         // half-frame limbs (0: v2 not used for this key size)
+  struct Half {
+    uint32_t n0inv;
+    size_t o_P, o_R2, o_R3;
+  } half[2];
+  H::Schedule sched_p, sched_q;           // exponents p and q
+  size_t o_sched_p = 0, o_sched_q = 0;
+  uint32_t n_n0inv = 0;
+  Blob blob;
+  DevBlob dev;
+  ~flb_priv() { delete pub; }
+};
+
+// A generic odd modulus for Table I's mod_mul / mod_pow and RSA (L247–L251): the
+// Montgomery constants live in an flb_pub "core" whose n2 slot holds the modulus, so the hom-add and
+// scalar-mul kernels serve mod_mul and per-element mod_pow unchanged.
+struct flb_mod {
+  flb_pub core;
+  std::mutex mu;
+  struct Sched {
+    H::Schedule s;
+    std::map<int, uint32_t*> dev;
+  };
+  std::map<std::vector<uint32_t>, Sched> scheds;  // batch-shared exponents seen so far
+  ~flb_mod() {
+    int cur;
+    if (cudaGetDevice(&cur) != cudaSuccess) return;
+    for (auto& kv : scheds)
+      for (auto& d : kv.second.dev) {
+        cudaSetDevice(d.first);
+        cudaFree(d.second);
+      }
+    cudaSetDevice(cur);
+  }
+};
+namespace flb_rt {
+
+// ----------------------------------------------------------------------------- launching
+struct Pool {
+  static int prepare() {
+    static std::mutex mu;
+    static std::map<int, bool> done;
+    int dev;
+    FLB_CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    if (!done[dev]) {
+      cudaMemPool_t pool;
+      FLB_CK(cudaDeviceGetDefaultMemPool(&pool, dev));
+      uint64_t thr = ~0ull;
+      FLB_CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+      done[dev] = true;
+    }
+    return FLB_OK;
+  }
+};
+
+template <typename K>
+inline int resident_blocks(K kernel, int* blocks) {
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, int> cache;
+  int dev;
+  FLB_CK(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair(dev, (const void*)kernel);
+  auto it = cache.find(key);
+  if (it != cache.end()) { *blocks = it->second; return FLB_OK; }
+  int per_sm = 0, sms = 0;
+  FLB_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kBlock, 0));
+  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  if (per_sm < 1) per_sm = 1;
+  cache[key] = per_sm * sms;
+  *blocks = per_sm * sms;
+  return FLB_OK;
+}
+
+// Grid for `items` work units of T lanes each: at most the resident capacity; the units are then
+// spread evenly over the rounds the persistent loop needs (ceil(items / capacity)), so the last
+// round is not a sliver of the grid — only with FLB_BALANCE=1: measured slower on B200 (fewer
+// resident warps cost more than the partial last round).
+inline bool balance_rounds() {
+  static bool v = [] {
+    const char* e = getenv("FLB_BALANCE");
+    return e && atoi(e) == 1;
+  }();
+  return v;
+}
+
+template <int T, typename K>
+inline int grid_for(K kernel, uint64_t items, int* grid) {
+  int cap;
+  int rc = resident_blocks(kernel, &cap);
+  if (rc) return rc;
+  const uint64_t per_block = kBlock / T;  // work units per block
+  const uint64_t cap_items = (uint64_t)cap * per_block;
+  uint64_t want = items;
+  if (items > cap_items) {
+    want = cap_items;
+    if (balance_rounds()) {
+      const uint64_t rounds = (items + cap_items - 1) / cap_items;
+      want = (items + rounds - 1) / rounds;
+    }
+  }
+  *grid = (int)std::max<uint64_t>(1, (want + per_block - 1) / per_block);
+  return FLB_OK;
+}
+
+struct Scratch {
+  void* p = nullptr;
+  cudaStream_t st = nullptr;
+  ~Scratch() {
+    if (p) cudaFreeAsync(p, st);
+  }
+  int alloc(size_t bytes, cudaStream_t s) {
+    st = s;
+    if (bytes == 0) return FLB_OK;
+    int rc = Pool::prepare();
+    if (rc) return rc;
+    FLB_CK(cudaMallocAsync(&p, bytes, s));
+    return FLB_OK;
+  }
+};
+
+#define FLB_LAUNCH_CHECK() FLB_CK(cudaGetLastError())
+
+// ---- encrypt
+template <int X, int T>
+int run_encrypt(const flb_pub* K, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)K->enc.table * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::EncArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.nR = dev + K->o_nR;
+  A.sched = dev + K->o_sched;
+  A.sched_len = (int)K->enc.ops.size();
+  A.table = K->enc.table;
+  A.nbits = K->nbits;
+  A.pt_words = K->sp;
+  A.m = m;
+  A.r = r;
+  A.c = c;
+  A.count = count;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_decrypt(const flb_priv* V, const uint32_t* dev, const uint32_t* c, uint32_t* m, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_decrypt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->pr[0].sched.table, V->pr[1].sched.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->pub->sp * 4, st);
+  if (rc) return rc;
+  flb::DecArgs A;
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    A.pr[i].P2 = {dev + R.o_P2, R.P2_n0inv};
+    A.pr[i].R2 = dev + R.o_R2;
+    A.pr[i].R3 = dev + R.o_R3;
+    A.pr[i].P = {dev + R.o_P, R.P_n0inv};
+    A.pr[i].Pinv = dev + R.o_Pinv;
+    A.pr[i].hR = dev + R.o_hR;
+    A.pr[i].sched = dev + R.o_sched;
+    A.pr[i].sched_len = (int)R.sched.ops.size();
+    A.pr[i].table = R.sched.table;
+  }
+  A.n = {dev + V->o_n, V->n_n0inv};
+  A.qR_n = dev + V->o_qR_n;
+  A.qinvR_p = dev + V->o_qinvR_p;
+  A.c = c;
+  A.m = m;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_decrypt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_encrypt_crt(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                    uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt_crt<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const flb_pub* K = V->pub;
+  Scratch sc;
+  rc = sc.alloc((size_t)K->enc.table * G * K->sp * 4, st);
+  if (rc) return rc;
+  flb::EncCrtArgs A;
+  for (int i = 0; i < 2; i++) {
+    A.P2[i] = {dev + V->pr[i].o_P2, V->pr[i].P2_n0inv};
+    A.R2[i] = dev + V->pr[i].o_R2;
+    A.nR[i] = dev + V->pr[i].o_nR;
+  }
+  A.q2 = dev + V->pr[1].o_P2;
+  A.q2invR = dev + V->o_q2invR;
+  A.sched = dev + V->o_enc_sched;
+  A.sched_len = (int)K->enc.ops.size();
+  A.table = K->enc.table;
+  A.nbits = K->nbits;
+  A.m = m;
+  A.r = r;
+  A.c = c;
+  A.count = count;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt_crt<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_modpow(const flb_pub* K, const uint32_t* dev, const uint32_t* sched, const H::Schedule* S, const uint32_t* base,
+               uint32_t* out, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_modpow<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)S->table * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::PowArgs A;
+  A.N = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.sched = sched;
+  A.sched_len = (int)S->ops.size();
+  A.table = S->table;
+  A.base = base;
+  A.out = out;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_modpow<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_horner(const flb_pub* K, const uint32_t* dev, const uint32_t* P, uint32_t planes, uint32_t* out, size_t nseg,
+               cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_horner<X, T>, nseg, &grid);
+  if (rc) return rc;
+  flb::HornerArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R1 = dev + K->o_R1;
+  A.R2 = dev + K->o_R2;
+  A.P = P;
+  A.K = planes;
+  A.out = out;
+  A.nseg = nseg;
+  flb::k_horner<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_mr(const uint32_t* cand, const uint32_t* bases, uint32_t rounds, uint64_t seed, uint64_t ctr0, uint32_t* verdict,
+           size_t count, int bw, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_miller_rabin<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  Scratch sc;
+  rc = sc.alloc((size_t)(1u << bw) * G * X * T * 4, st);
+  if (rc) return rc;
+  flb::MrArgs A;
+  A.cand = cand;
+  A.bases = bases;
+  A.rounds = rounds;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.verdict = verdict;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  A.bw = bw;
+  flb::k_miller_rabin<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_crt_pre(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* y,
+                size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_crt_pre<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->sched_p.table, V->sched_q.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->H * 4, st);
+  if (rc) return rc;
+  flb::CrtPreArgs A;
+  for (int i = 0; i < 2; i++) {
+    A.P[i] = {dev + V->half[i].o_P, V->half[i].n0inv};
+    A.R2[i] = dev + V->half[i].o_R2;
+    A.R3[i] = dev + V->half[i].o_R3;
+    const H::Schedule& sc_i = i == 0 ? V->sched_q : V->sched_p;  // exponent: the other prime
+    A.sched[i] = dev + (i == 0 ? V->o_sched_q : V->o_sched_p);
+    A.sched_len[i] = (int)sc_i.ops.size();
+    A.table[i] = sc_i.table;
+  }
+  A.nbits = V->pub->nbits;
+  A.pt_words = V->pub->sp;
+  A.r = r;
+  A.seed = seed;
+  A.ctr0 = ctr0;
+  A.y = y;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_crt_pre<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_encrypt_crt2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
+                     size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_encrypt_crt2<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const int table = std::max(V->sched_p.table, V->sched_q.table);
+  Scratch sc;
+  rc = sc.alloc((size_t)table * G * V->pub->sp * 4, st);
+  if (rc) return rc;
+  flb::EncCrt2Args A;
+  for (int i = 0; i < 2; i++) {
+    A.P2[i] = {dev + V->pr[i].o_P2, V->pr[i].P2_n0inv};
+    A.R2[i] = dev + V->pr[i].o_R2;
+    A.nR[i] = dev + V->pr[i].o_nR;
+    const H::Schedule& sc_i = i == 0 ? V->sched_p : V->sched_q;  // exponent P for P^2
+    A.sched[i] = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
+    A.sched_len[i] = (int)sc_i.ops.size();
+    A.table[i] = sc_i.table;
+  }
+  A.q2 = dev + V->pr[1].o_P2;
+  A.q2invR = dev + V->o_q2invR;
+  A.m = m;
+  A.y = y;
+  A.H = V->H;
+  A.c = c;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_encrypt_crt2<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T, bool DEBUG>
+int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
+            cudaStream_t st) {
+  auto kern = DEBUG ? flb::k_mont<X, T> : flb::k_add<X, T>;
+  int grid;
+  int rc = grid_for<T>(kern, count, &grid);
+  if (rc) return rc;
+  flb::AddArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.c1 = a;
+  A.c2 = b;
+  A.out = out;
+  A.count = count;
+  kern<<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_smul(const flb_pub* K, const uint32_t* dev, const uint32_t* c, const uint32_t* e, uint32_t e_words,
+             uint32_t* out, size_t count, cudaStream_t st) {
+  int grid;
+  int rc = grid_for<T>(flb::k_scalar_mul<X, T>, count, &grid);
+  if (rc) return rc;
+  const uint64_t G = (uint64_t)grid * kBlock / T;
+  const uint32_t ebits = 32 * e_words;
+  const int bw = ebits <= 64 ? 3 : (ebits <= 512 ? 5 : 6);
+  Scratch sc;
+  rc = sc.alloc((size_t)(1u << bw) * G * K->s * 4, st);
+  if (rc) return rc;
+  flb::SmulArgs A;
+  A.N2 = {dev + K->o_n2, K->n2_n0inv};
+  A.R2 = dev + K->o_R2;
+  A.R1 = dev + K->o_R1;
+  A.c = c;
+  A.e = e;
+  A.e_words = e_words;
+  A.bw = bw;
+  A.out = out;
+  A.count = count;
+  A.scratch = (uint32_t*)sc.p;
+  flb::k_scalar_mul<X, T><<<grid, kBlock, 0, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+template <int X, int T>
+int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t num_entries, const int64_t* idx,
+               const int64_t* offsets, size_t nseg, size_t max_len, uint32_t* out, cudaStream_t st) {
+  const int C = kReduceChunk;
+  const size_t num_inputs = num_entries;  // chunk bounds follow the entries (idx may repeat inputs)
+  if (max_len == 0 || max_len > num_entries) max_len = std::max<size_t>(num_entries, 1);
+  int levels = 1;
+  for (size_t cap = C; cap < max_len; cap *= C) levels++;
+  // per-level buffers: chunk offsets [nseg+1], starts/ends [max_chunks], partials
+  const size_t max_chunks0 = num_inputs / C + nseg + 1;
+  Scratch s_plan, s_part0, s_part1;
+  const size_t plan_words = (nseg + 1) + 2 * max_chunks0;
+  int rc = s_plan.alloc(plan_words * sizeof(int64_t), st);
+  if (rc) return rc;
+  int64_t* chunk_off = (int64_t*)s_plan.p;
+  int64_t* cstart = chunk_off + (nseg + 1);
+  int64_t* cend = cstart + max_chunks0;
+  // partial buffers (ping-pong), sized for level 0 output
+  if (levels > 1) {
+    rc = s_part0.alloc(max_chunks0 * K->s * 4, st);
+    if (rc) return rc;
+    if (levels > 2) {
+      rc = s_part1.alloc((max_chunks0 / C + nseg + 1) * K->s * 4, st);
+      if (rc) return rc;
+    }
+  }
+  int grid_r;
+  rc = grid_for<T>(flb::k_reduce<X, T>, max_chunks0, &grid_r);
+  if (rc) return rc;
+  const uint32_t* in = c;
+  const int64_t* cur_idx = idx;
+  const int64_t* cur_off = offsets;
+  // level-(>0) offsets must survive while the next plan is built: keep two offset arrays
+  Scratch s_off;
+  rc = s_off.alloc(2 * (nseg + 1) * sizeof(int64_t), st);
+  if (rc) return rc;
+  int64_t* offbuf[2] = {(int64_t*)s_off.p, (int64_t*)s_off.p + (nseg + 1)};
+  size_t in_chunks = max_chunks0;
+  for (int lv = 0; lv < levels; lv++) {
+    flb::k_plan_scan<<<1, 1024, 0, st>>>(cur_off, (int64_t)nseg, C, chunk_off);
+    FLB_LAUNCH_CHECK();
+    const int fill_grid = (int)std::min<size_t>(4096, (in_chunks + 255) / 256 + 1);
+    flb::k_plan_fill<<<fill_grid, 256, 0, st>>>(cur_off, chunk_off, (int64_t)nseg, C, cstart, cend);
+    FLB_LAUNCH_CHECK();
+    const bool last = lv == levels - 1;
+    uint32_t* dst = last ? out : (uint32_t*)((lv % 2 == 0) ? s_part0.p : s_part1.p);
+    flb::RedArgs A;
+    A.N2 = {dev + K->o_n2, K->n2_n0inv};
+    A.R1 = dev + K->o_R1;
+    A.RL = dev + K->o_RL;
+    A.in = in;
+    A.idx = cur_idx;
+    A.cstart = cstart;
+    A.cend = cend;
+    A.nchunks = chunk_off + nseg;
+    A.out = dst;
+    A.max_chunks = in_chunks;
+    flb::k_reduce<X, T><<<grid_r, kBlock, 0, st>>>(A);
+    FLB_LAUNCH_CHECK();
+    if (!last) {
+      // next level: segments over this level's chunk partials
+      int64_t* nxt = offbuf[lv % 2];
+      FLB_CK(cudaMemcpyAsync(nxt, chunk_off, (nseg + 1) * sizeof(int64_t), cudaMemcpyDeviceToDevice, st));
+      cur_off = nxt;
+      in = dst;
+      cur_idx = nullptr;
+      in_chunks = in_chunks / C + nseg + 1;
+    }
+  }
+  return FLB_OK;
+}
+
+}  // namespace flb_rt
+
+// ----------------------------------------------------------------------------- instantiation lists
+// (X, T) splits used by the dispatch macros of flb_api.cu: ENC frames run the public-key / generic
+// kernels, DEC frames the private-key kernels (sp-limb frames).
+#define FLB_ENC_COMBOS(M) M(16, 2) M(16, 4) M(8, 8) M(12, 8) M(16, 8) M(8, 16) M(12, 16) M(16, 16) M(8, 32)
+#define FLB_DEC_COMBOS(M) M(16, 2) M(8, 4) M(16, 4) M(8, 8) M(12, 8) M(16, 8) M(8, 16)
+
+#define FLB_ENC_DECLS(EXT, X, T)                                                                                  \
+  EXT template int flb_rt::run_encrypt<X, T>(const flb_pub*, const uint32_t*, const uint32_t*, const uint32_t*,  \
+                                             uint64_t, uint64_t, uint32_t*, size_t, cudaStream_t);                \
+  EXT template int flb_rt::run_modpow<X, T>(const flb_pub*, const uint32_t*, const uint32_t*,                     \
+                                            const flb::host::Schedule*, const uint32_t*, uint32_t*, size_t,       \
+                                            cudaStream_t);                                                        \
+  EXT template int flb_rt::run_horner<X, T>(const flb_pub*, const uint32_t*, const uint32_t*, uint32_t, uint32_t*, \
+                                            size_t, cudaStream_t);                                                \
+  EXT template int flb_rt::run_mr<X, T>(const uint32_t*, const uint32_t*, uint32_t, uint64_t, uint64_t, uint32_t*, \
+                                        size_t, int, cudaStream_t);                                               \
+  EXT template int flb_rt::run_crt_pre<X, T>(const flb_priv*, const uint32_t*, const uint32_t*, uint64_t, uint64_t, \
+                                             uint32_t*, size_t, cudaStream_t);                                    \
+  EXT template int flb_rt::run_add<X, T, false>(const flb_pub*, const uint32_t*, const uint32_t*, const uint32_t*, \
+                                                uint32_t*, size_t, cudaStream_t);                                 \
+  EXT template int flb_rt::run_add<X, T, true>(const flb_pub*, const uint32_t*, const uint32_t*, const uint32_t*,  \
+                                               uint32_t*, size_t, cudaStream_t);                                  \
+  EXT template int flb_rt::run_smul<X, T>(const flb_pub*, const uint32_t*, const uint32_t*, const uint32_t*,      \
+                                          uint32_t, uint32_t*, size_t, cudaStream_t);                             \
+  EXT template int flb_rt::run_reduce<X, T>(const flb_pub*, const uint32_t*, const uint32_t*, size_t,              \
+                                            const int64_t*, const int64_t*, size_t, size_t, uint32_t*,            \
+                                            cudaStream_t);
+#define FLB_DEC_DECLS(EXT, X, T)                                                                                  \
+  EXT template int flb_rt::run_decrypt<X, T>(const flb_priv*, const uint32_t*, const uint32_t*, uint32_t*, size_t, \
+                                             cudaStream_t);                                                       \
+  EXT template int flb_rt::run_encrypt_crt<X, T>(const flb_priv*, const uint32_t*, const uint32_t*,              \
+                                                 const uint32_t*, uint64_t, uint64_t, uint32_t*, size_t,          \
+                                                 cudaStream_t);                                                   \
+  EXT template int flb_rt::run_encrypt_crt2<X, T>(const flb_priv*, const uint32_t*, const uint32_t*,             \
+                                                  const uint32_t*, uint32_t*, size_t, cudaStream_t);
+
+#ifndef FLB_INST_TU
+#define FLB_EXTERN_ENC(X, T) FLB_ENC_DECLS(extern, X, T)
+#define FLB_EXTERN_DEC(X, T) FLB_DEC_DECLS(extern, X, T)
+FLB_ENC_COMBOS(FLB_EXTERN_ENC)
+FLB_DEC_COMBOS(FLB_EXTERN_DEC)
+#undef FLB_EXTERN_ENC
+#undef FLB_EXTERN_DEC
+#endif

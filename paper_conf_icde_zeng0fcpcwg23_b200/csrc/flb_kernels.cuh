@@ -394,7 +394,7 @@ __global__ void __launch_bounds__(32, FLB_MINB_ENC) k_modpow(const PowArgs A) {
 }
 
 // out[i] = 1 (the empty product / x^0), [count][S]
-__global__ void k_fill_one(uint32_t* out, uint64_t count, uint32_t S) {
+static __global__ void k_fill_one(uint32_t* out, uint64_t count, uint32_t S) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count * S; i += (uint64_t)gridDim.x * blockDim.x)
     out[i] = (i % S) == 0 ? 1u : 0u;
 }
@@ -542,7 +542,7 @@ __global__ void __launch_bounds__(32, FLB_MINB_ENC) k_miller_rabin(const MrArgs 
 
 // candidates for key generation: Philox words, bits above `bits` cleared, top two bits and bit 0
 // set (reading c5), limbs above the prime's words zero; one thread per limb.
-__global__ void k_gen_candidates(uint32_t* cand, uint64_t count, uint32_t S, uint32_t bits, uint64_t seed,
+static __global__ void k_gen_candidates(uint32_t* cand, uint64_t count, uint32_t S, uint32_t bits, uint64_t seed,
                                  uint64_t ctr0) {
   const uint64_t total = count * S;
   for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < total; t += (uint64_t)gridDim.x * blockDim.x) {
@@ -565,7 +565,7 @@ __global__ void k_gen_candidates(uint32_t* cand, uint64_t count, uint32_t S, uin
 }
 
 // small-prime sieve: flag[i] = 1 if no prime in `primes` divides candidate i
-__global__ void k_sieve(const uint32_t* __restrict__ cand, uint64_t count, uint32_t S, uint32_t words,
+static __global__ void k_sieve(const uint32_t* __restrict__ cand, uint64_t count, uint32_t S, uint32_t words,
                         const uint32_t* __restrict__ primes, uint32_t nprimes, uint32_t* __restrict__ flag) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t* c = cand + i * S;
@@ -624,7 +624,7 @@ __global__ void k_bucket(const int64_t* __restrict__ off, int64_t nseg, int64_t 
 }
 
 // exclusive scan of n counters (one block): out[i] = sum_{k<i} in[k], out[n] = total
-__global__ void k_scan_u64(const unsigned long long* __restrict__ in, int64_t n, int64_t* __restrict__ out) {
+static __global__ void k_scan_u64(const unsigned long long* __restrict__ in, int64_t n, int64_t* __restrict__ out) {
   __shared__ long long warp_sums[32];
   __shared__ long long carry;
   if (threadIdx.x == 0) carry = 0;
@@ -661,7 +661,7 @@ __global__ void k_scan_u64(const unsigned long long* __restrict__ in, int64_t n,
 }
 
 // bit-plane index: for plane p = (j, w, bit) list the buckets (j, w, v) with that bit of v set
-__global__ void k_bitplane_index(int64_t nplanes, uint32_t cb, int64_t* __restrict__ idx2) {
+static __global__ void k_bitplane_index(int64_t nplanes, uint32_t cb, int64_t* __restrict__ idx2) {
   const int64_t half = (int64_t)1 << (cb - 1);
   const int64_t total = nplanes * half;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
@@ -675,7 +675,7 @@ __global__ void k_bitplane_index(int64_t nplanes, uint32_t cb, int64_t* __restri
   }
 }
 
-__global__ void k_arange_offsets(int64_t n, int64_t step, int64_t* __restrict__ out) {
+static __global__ void k_arange_offsets(int64_t n, int64_t step, int64_t* __restrict__ out) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
     out[i] = i * step;
 }
@@ -718,7 +718,7 @@ __global__ void __launch_bounds__(32, FLB_MINB_MUL) k_horner(const HornerArgs A)
 }
 
 // rows[i] = c[idx[i]] (gather, one thread per word)
-__global__ void k_gather_rows(const uint32_t* __restrict__ c, const int64_t* __restrict__ idx, int64_t n, uint32_t S,
+static __global__ void k_gather_rows(const uint32_t* __restrict__ c, const int64_t* __restrict__ idx, int64_t n, uint32_t S,
                               uint32_t* __restrict__ out) {
   const int64_t total = n * S;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
@@ -1033,7 +1033,7 @@ __global__ void __launch_bounds__(32, FLB_MINB_MUL) k_reduce(const RedArgs A) {
 }
 
 // chunk planning: chunks_j = max(1, ceil(len_j / C)); chunk_off = exclusive scan (one block).
-__global__ void k_plan_scan(const int64_t* __restrict__ offsets, int64_t nseg, int C, int64_t* __restrict__ chunk_off) {
+static __global__ void k_plan_scan(const int64_t* __restrict__ offsets, int64_t nseg, int C, int64_t* __restrict__ chunk_off) {
   __shared__ int64_t warp_sums[32];
   __shared__ int64_t carry;
   if (threadIdx.x == 0) carry = 0;
@@ -1074,7 +1074,7 @@ __global__ void k_plan_scan(const int64_t* __restrict__ offsets, int64_t nseg, i
   if (threadIdx.x == 0) chunk_off[nseg] = carry;
 }
 
-__global__ void k_plan_fill(const int64_t* __restrict__ offsets, const int64_t* __restrict__ chunk_off, int64_t nseg,
+static __global__ void k_plan_fill(const int64_t* __restrict__ offsets, const int64_t* __restrict__ chunk_off, int64_t nseg,
                             int C, int64_t* __restrict__ cstart, int64_t* __restrict__ cend) {
   const int64_t total = chunk_off[nseg];
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < total; c += (int64_t)gridDim.x * blockDim.x) {
@@ -1115,7 +1115,7 @@ __device__ __forceinline__ uint64_t quantize(float xf, const CodecArgs& C) {
 }
 
 // pt[j] = sum_i q_{jS+i} 2^((S-1-i) w) (Eq. 9, reading c17); one thread per word.
-__global__ void k_pack(const float* __restrict__ x, uint64_t n_values, uint64_t n_pt, CodecArgs C,
+static __global__ void k_pack(const float* __restrict__ x, uint64_t n_values, uint64_t n_pt, CodecArgs C,
                        uint32_t* __restrict__ pt) {
   const uint64_t total = n_pt * C.pt_words;
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -1142,7 +1142,7 @@ __device__ __forceinline__ uint64_t slot_value(const uint32_t* __restrict__ pt, 
 }
 
 // x = Sum / sigma - cnt alpha in binary64, then binary32 (reading c14).
-__global__ void k_unpack(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
+static __global__ void k_unpack(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
                          const uint32_t* __restrict__ summands, uint32_t summands_scalar, float* __restrict__ out) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n_values; v += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t s = slot_value(pt, v, C);
@@ -1153,7 +1153,7 @@ __global__ void k_unpack(const uint32_t* __restrict__ pt, uint64_t n_values, Cod
   }
 }
 
-__global__ void k_unpack_sums(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
+static __global__ void k_unpack_sums(const uint32_t* __restrict__ pt, uint64_t n_values, CodecArgs C,
                               unsigned long long* __restrict__ out) {
   for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n_values; v += (uint64_t)gridDim.x * blockDim.x)
     out[v] = slot_value(pt, v, C);

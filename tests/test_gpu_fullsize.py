@@ -134,3 +134,21 @@ def test_roundtrip_beyond_one_wave(name, count):
     for i in (0, count - 1):
         assert synthetic.limbs_to_ints(cl[i:i + 1])[0] == paillier.encrypt(n, ms[i],
                                                                           philox.draw_r(n, 3, i, pub.pt_words))
+
+
+def test_c2_full_batch_public_equals_keyholder(key2048):
+    """Every one of the bench's 133,160 ciphertexts agrees between the public-key path (n^2 frame,
+    8 lanes per integer, exponent n) and the two-stage key-holder path (half and p^2 frames, 2 and 4
+    lanes, exponents q then p): independent operand sets, so a rare carry slip in either shows up
+    here even when sampled oracle checks miss it (a one-in-2^30-steps carry bug did, in development)."""
+    pub, priv, p, q = key2048
+    count = 133160
+    g = torch.Generator().manual_seed(2048)
+    m = torch.randint(-2**31, 2**31 - 1, (count, pub.pt_words), generator=g, dtype=torch.int32)
+    m[:, -1] &= 0x3FFFFFFF  # m < 2^2046 < n
+    m = m.cuda()
+    a = flb.encrypt(pub, m, seed=0xC2000001)
+    b = flb.encrypt_crt(priv, m, seed=0xC2000001)
+    bad = (a != b).any(dim=1).nonzero().flatten().tolist()
+    assert not bad, f"{len(bad)} of {count} ciphertexts differ, first {bad[:5]}"
+    assert torch.equal(flb.decrypt(priv, b), m)
