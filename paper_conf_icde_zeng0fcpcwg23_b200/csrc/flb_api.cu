@@ -111,6 +111,46 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
       V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
     }
   }
+  // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 frames of 1024- and 2048-bit keys:
+  // B1[n][k] = N'_(n-k) (N' = -N^-1 mod R), B2h[n][k] = N_(KB+n-k), B2b[j][k] = N_(KB-16+j-k), bytes,
+  // zero outside the band, in the K-major core-matrix layout the MMA descriptors describe
+  if (sp == 32 || sp == 64) {
+    const uint32_t KB = 4 * sp, kch = KB / 16;
+    auto bytes_of = [](const Limbs& v, size_t nbytes) {
+      std::vector<uint8_t> b(nbytes, 0);
+      for (size_t i = 0; i < nbytes && i / 4 < v.size(); i++) b[i] = (uint8_t)(v[i / 4] >> (8 * (i % 4)));
+      return b;
+    };
+    auto put_bytes = [&](const std::vector<uint8_t>& m) {
+      std::vector<uint32_t> w((m.size() + 3) / 4, 0);
+      for (size_t i = 0; i < m.size(); i++) w[i / 4] |= (uint32_t)m[i] << (8 * (i % 4));
+      return V->blob.put_raw(w);
+    };
+    for (int i = 0; i < 2; i++) {
+      auto& R = V->pr[i];
+      Limbs inv = H::inv_mod_2k(R.P2, sp);  // N^-1 mod R
+      Limbs np = H::resized(inv, sp);        // N' = R - N^-1 = two's complement of N^-1 mod R
+      uint64_t cy = 1;
+      for (auto& w : np) { cy += (uint32_t)~w; w = (uint32_t)cy; cy >>= 32; }
+      const std::vector<uint8_t> nb = bytes_of(R.P2, KB), npb = bytes_of(np, KB);
+      std::vector<uint8_t> b1((size_t)KB * KB, 0), b2h((size_t)KB * KB, 0), b2b((size_t)16 * KB, 0);
+      for (uint32_t n = 0; n < KB; n++)
+        for (uint32_t k = 0; k < KB; k++) {
+          if (k <= n) b1[flb::tc::cm_off(n, k, kch)] = npb[n - k];
+          const int64_t d = (int64_t)KB + n - k;
+          if (d >= 0 && d < (int64_t)KB) b2h[flb::tc::cm_off(n, k, kch)] = nb[d];
+        }
+      for (uint32_t j = 0; j < 16; j++)
+        for (uint32_t k = 0; k < KB; k++) {
+          const int64_t d = (int64_t)KB - 16 + j - k;
+          if (d >= 0 && d < (int64_t)KB) b2b[flb::tc::cm_off(j, k, kch)] = nb[d];
+        }
+      R.o_tcB1 = put_bytes(b1);
+      R.o_tcB2h = put_bytes(b2h);
+      R.o_tcB2b = put_bytes(b2b);
+    }
+    V->tc = true;
+  }
   // CRT recombination constants
   H::MontCtx Cn(V->pub->n), Cp(V->p);
   V->n_n0inv = Cn.n0inv;
@@ -619,6 +659,14 @@ static int crt2_dispatch(const flb_priv* V, const uint32_t* dev, const uint32_t*
   FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt2, V, dev, m, y, c, count, st);
 }
 
+// tensor-core Montgomery path for the key-holder stage 2 (flb_tc.cuh): on when the key has the
+// operands; FLB_TC=0 selects the CIOS kernel (read per call, so tests can compare both)
+static bool use_tc(const flb_priv* V) {
+  if (!V->tc) return false;
+  const char* e = getenv("FLB_TC");
+  return !(e && atoi(e) == 0);
+}
+
 static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
                           uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
   Scratch ys;
@@ -626,6 +674,10 @@ static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t
   if (rc) return rc;
   rc = crt_pre_dispatch(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
   if (rc) return rc;
+  if (use_tc(V)) {
+    if (V->pub->sp == 64) return run_encrypt_crt_tc<64>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
+    return run_encrypt_crt_tc<32>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
+  }
   return crt2_dispatch(V, dev, m, (const uint32_t*)ys.p, c, count, st);
 }
 

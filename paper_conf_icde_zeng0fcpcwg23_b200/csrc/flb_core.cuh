@@ -18,6 +18,7 @@
 
 #include "../../include/flb_paillier.h"
 #include "flb_kernels.cuh"
+#include "flb_tc.cuh"
 #include "host_bn.hpp"
 
 using flb::host::Limbs;
@@ -122,7 +123,10 @@ struct flb_priv {
     H::Schedule sched;
     size_t o_P, o_P2, o_R2, o_R3, o_Pinv, o_hR, o_sched;
     size_t o_nR;  // n R mod P^2 (key-holder encryption)
+    // tensor-core Montgomery operands for P^2 (flb_tc.cuh), core-matrix byte layout; 0 = absent
+    size_t o_tcB1 = 0, o_tcB2h = 0, o_tcB2b = 0;
   } pr[2];
+  bool tc = false;  // tc operands present (sp in {32, 64})
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
   size_t o_q2invR = 0, o_enc_sched = 0;  // key-holder encryption: (q^2)^-1 R mod p^2, schedule of n
   // key-holder encryption v2 (r^n mod P^2 = (r^Q mod P)^P mod P^2): half-frame moduli and schedules
@@ -489,6 +493,68 @@ int run_encrypt_crt2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, 
   return FLB_OK;
 }
 
+// key-holder stage 2 with the Montgomery reductions on the tensor cores (flb_tc.cuh): c_p and c_q
+// by k_tc_pow (one launch per prime), then k_crt_combine.
+template <int S>
+int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
+                       size_t count, cudaStream_t st) {
+  using C = flb::tc::Cfg<S>;
+  static bool attr_done = false;
+  if (!attr_done) {
+    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_pow<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+    attr_done = true;
+  }
+  int sms = 0, dev_id = 0;
+  FLB_CK(cudaGetDevice(&dev_id));
+  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id));
+  const uint64_t tiles = (count + flb::tc::kTileM - 1) / flb::tc::kTileM;
+  const int grid = (int)std::min<uint64_t>((uint64_t)sms, tiles);
+  const int table = std::max(V->sched_p.table, V->sched_q.table);
+  Scratch s_out, s_tab;
+  int rc = s_out.alloc((size_t)2 * count * S * 4, st);
+  if (rc) return rc;
+  rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
+  if (rc) return rc;
+  uint32_t* cpq = (uint32_t*)s_out.p;
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    const H::Schedule& sc = i == 0 ? V->sched_p : V->sched_q;  // exponent P for P^2
+    flb::tc::PowArgs A;
+    A.P2 = dev + R.o_P2;
+    A.R2 = dev + R.o_R2;
+    A.nR = dev + R.o_nR;
+    A.B1 = dev + R.o_tcB1;
+    A.B2h = dev + R.o_tcB2h;
+    A.B2b = dev + R.o_tcB2b;
+    A.sched = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
+    A.sched_len = (int)sc.ops.size();
+    A.table = sc.table;
+    A.y = y + (size_t)i * count * V->H;
+    A.H = V->H;
+    A.m = m;
+    A.out = cpq + (size_t)i * count * S;
+    A.count = count;
+    A.scratch = (uint32_t*)s_tab.p;
+    flb::tc::k_tc_pow<S><<<grid, flb::tc::kThreads, C::SMEM, st>>>(A);
+    FLB_LAUNCH_CHECK();
+  }
+  constexpr int XC = 16, TC = S / 16;
+  int cgrid;
+  rc = grid_for<TC>(flb::k_crt_combine<XC, TC>, count, &cgrid);
+  if (rc) return rc;
+  flb::CombineArgs B;
+  B.P2 = {dev + V->pr[0].o_P2, V->pr[0].P2_n0inv};
+  B.q2 = dev + V->pr[1].o_P2;
+  B.q2invR = dev + V->o_q2invR;
+  B.cp = cpq;
+  B.cq = cpq + (size_t)count * S;
+  B.c = c;
+  B.count = count;
+  flb::k_crt_combine<XC, TC><<<cgrid, kBlock, 0, st>>>(B);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
 template <int X, int T, bool DEBUG>
 int run_add(const flb_pub* K, const uint32_t* dev, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
             cudaStream_t st) {
@@ -645,12 +711,17 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
                                                  cudaStream_t);                                                   \
   EXT template int flb_rt::run_encrypt_crt2<X, T>(const flb_priv*, const uint32_t*, const uint32_t*,             \
                                                   const uint32_t*, uint32_t*, size_t, cudaStream_t);
+#define FLB_TC_DECLS(EXT, S)                                                                                      \
+  EXT template int flb_rt::run_encrypt_crt_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*,              \
+                                                 const uint32_t*, uint32_t*, size_t, cudaStream_t);
 
 #ifndef FLB_INST_TU
 #define FLB_EXTERN_ENC(X, T) FLB_ENC_DECLS(extern, X, T)
 #define FLB_EXTERN_DEC(X, T) FLB_DEC_DECLS(extern, X, T)
 FLB_ENC_COMBOS(FLB_EXTERN_ENC)
 FLB_DEC_COMBOS(FLB_EXTERN_DEC)
+FLB_TC_DECLS(extern, 32)
+FLB_TC_DECLS(extern, 64)
 #undef FLB_EXTERN_ENC
 #undef FLB_EXTERN_DEC
 #endif

@@ -11,3 +11,21 @@ FLB_ENC_DECLS(, FLB_INST_X, FLB_INST_T)
 #if FLB_INST_DEC
 FLB_DEC_DECLS(, FLB_INST_X, FLB_INST_T)
 #endif
+#if defined(FLB_INST_TC)
+FLB_TC_DECLS(, FLB_INST_TC)
+#endif
+
+#if defined(FLB_INST_TC) && FLB_INST_TC == 64 && FLB_TC_PROF
+// profiling builds only (FLB_NVCC_EXTRA=-DFLB_TC_PROF=1; not in include/): per-phase cycle totals of
+// thread 0 of the 2048-bit tensor-core Montgomery kernel (tools/tc_phases.py)
+extern "C" int flb_debug_tc_prof(uint64_t* out8, int reset) {
+  unsigned long long h[8];
+  FLB_CK(cudaMemcpyFromSymbol(h, flb::tc::g_tc_prof, sizeof(h)));
+  for (int i = 0; i < 8; i++) out8[i] = h[i];
+  if (reset) {
+    unsigned long long z[8] = {};
+    FLB_CK(cudaMemcpyToSymbol(flb::tc::g_tc_prof, z, sizeof(z)));
+  }
+  return FLB_OK;
+}
+#endif

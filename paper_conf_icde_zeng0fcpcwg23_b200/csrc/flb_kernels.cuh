@@ -1160,3 +1160,46 @@ static __global__ void k_unpack_sums(const uint32_t* __restrict__ pt, uint64_t n
 }
 
 }  // namespace flb
+
+namespace flb {
+// ----------------------------------------------------------------------------- CRT combine
+// c = c_q + q^2 ((c_p - c_q) (q^2)^-1 mod p^2) from c_p = c mod p^2, c_q = c mod q^2 (the combine
+// step of k_encrypt_crt2, for stage-2 results computed elsewhere, e.g. by the tensor-core kernel).
+struct CombineArgs {
+  ModRef P2;               // p^2 in the sp frame
+  const uint32_t* q2;      // q^2 (sp limbs, plain)
+  const uint32_t* q2invR;  // (q^2)^-1 R mod p^2
+  const uint32_t* cp;      // [count][sp]
+  const uint32_t* cq;      // [count][sp]
+  uint32_t* c;             // [count][2 sp]
+  uint64_t count;
+};
+
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_crt_combine(const CombineArgs A) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t n[X], d[X], t[X], hi[X], cp[X], cq[X];
+    load_elem<X, T>(cp, A.cp + e * S, S, valid);
+    load_elem<X, T>(cq, A.cq + e * S, S, valid);
+    load_mod<X, T>(n, A.P2);
+    const uint32_t br = grp_sub<X, T>(d, cp, cq);
+#pragma unroll
+    for (int j = 0; j < X; j++) t[j] = br ? n[j] : 0u;
+    grp_add<X, T>(d, d, t);
+    load_const<X, T>(t, A.q2invR);
+    mont_mul<X, T>(d, d, t, n, A.P2.n0inv);
+    load_const<X, T>(t, A.q2);
+    mul_full<X, T>(d, hi, d, t);
+    const uint32_t cy = grp_add<X, T>(d, d, cq);
+    grp_add_small<X, T>(hi, cy);
+    if (valid) {
+      store_limbs<X>(A.c + e * (2 * S) + g.k * X, d);
+      store_limbs<X>(A.c + e * (2 * S) + S + g.k * X, hi);
+    }
+  }
+}
+}  // namespace flb

@@ -34,9 +34,19 @@ def timed(fn, reps=3):
 
 
 out = {"lib": flb.library_path, "bits": bits, "count": count}
+os.environ["FLB_TC"] = "0"
 c = flb.encrypt_crt(priv, m, seed=3)
 t = timed(lambda: flb.encrypt_crt(priv, m, seed=3))
 out["encrypt_keyholder_per_s"] = count / t
+os.environ["FLB_TC"] = "1"
+ctc = flb.encrypt_crt(priv, m, seed=3)
+torch.cuda.synchronize()
+bad = (ctc != c).any(dim=1).nonzero().flatten().tolist()
+out["tc_mismatches"] = len(bad)
+out["tc_first_bad"] = bad[:3]
+t = timed(lambda: flb.encrypt_crt(priv, m, seed=3))
+out["encrypt_keyholder_tc_per_s"] = count / t
+os.environ["FLB_TC"] = "0"
 t = timed(lambda: flb.encrypt(pub, m, seed=3), reps=1)
 out["encrypt_public_per_s"] = count / t
 t = timed(lambda: flb.decrypt(priv, c))

@@ -1,0 +1,30 @@
+"""Per-phase cycles of the tensor-core Montgomery kernel (thread 0 of each CTA, summed), from a
+FLB_TC_PROF=1 build:  FLB_LIB_PATH=build_variants/tcprof.so python tools/tc_phases.py [count]"""
+import ctypes
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import paper_conf_icde_zeng0fcpcwg23_b200 as flb  # noqa: E402
+
+count = int(sys.argv[1]) if len(sys.argv) > 1 else 18944
+pub, priv = flb.keygen(2048, 0xF1B0 + 2048)
+m = torch.randint(0, 2**31 - 1, (count, 64), dtype=torch.int32).cuda()
+fn = flb.LIB.flb_debug_tc_prof
+fn.argtypes = [ctypes.POINTER(ctypes.c_uint64), ctypes.c_int]
+buf = (ctypes.c_uint64 * 8)()
+flb.encrypt_crt(priv, m, seed=1)
+torch.cuda.synchronize()
+fn(buf, 1)
+flb.encrypt_crt(priv, m, seed=1)
+torch.cuda.synchronize()
+fn(buf, 0)
+calls = buf[5]
+names = ["P (product + sA/t_hi writes + barrier)", "M1 issue + wait", "N1 (q normalise + resolve + sA)",
+         "M2 wait", "F (finish + borrow + writes)"]
+tot = sum(buf[i] for i in range(5))
+print(json.dumps({"calls": calls, "cycles_per_call": tot / max(calls, 1),
+                  "phases": {n: round(buf[i] / max(calls, 1)) for i, n in enumerate(names)}}, indent=1))
