@@ -112,42 +112,34 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
     }
   }
   // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 frames of 1024- and 2048-bit keys:
-  // B1[n][k] = N'_(n-k) (N' = -N^-1 mod R), B2h[n][k] = N_(KB+n-k), B2b[j][k] = N_(KB-16+j-k), bytes,
-  // zero outside the band, in the K-major core-matrix layout the MMA descriptors describe
-  if (sp == 32 || sp == 64) {
-    const uint32_t KB = 4 * sp, kch = KB / 16;
+  // extended Toeplitz K-slices Ext[r][kk] = V_(r - KB - kk) (bytes, zero outside [0, KB)) of
+  // V = N' = -N^-1 mod R (2 KB rows) and V = N (3 KB rows), 32 bytes per row, in the K-major
+  // core-matrix layout the MMA descriptors describe
+  if ((sp == 32 || sp == 64) && V->H) {
+    const uint32_t KB = 4 * sp;
     auto bytes_of = [](const Limbs& v, size_t nbytes) {
       std::vector<uint8_t> b(nbytes, 0);
       for (size_t i = 0; i < nbytes && i / 4 < v.size(); i++) b[i] = (uint8_t)(v[i / 4] >> (8 * (i % 4)));
       return b;
     };
-    auto put_bytes = [&](const std::vector<uint8_t>& m) {
-      std::vector<uint32_t> w((m.size() + 3) / 4, 0);
+    auto ext = [&](const std::vector<uint8_t>& vb, uint32_t rows) {
+      std::vector<uint8_t> m((size_t)rows * 32, 0);
+      for (uint32_t r = 0; r < rows; r++)
+        for (uint32_t kk = 0; kk < 32; kk++) {
+          const int64_t d = (int64_t)r - KB - kk;
+          if (d >= 0 && d < (int64_t)KB) m[flb::tc::cm_off(r, kk, 2)] = vb[d];
+        }
+      std::vector<uint32_t> w(m.size() / 4, 0);
       for (size_t i = 0; i < m.size(); i++) w[i / 4] |= (uint32_t)m[i] << (8 * (i % 4));
       return V->blob.put_raw(w);
     };
     for (int i = 0; i < 2; i++) {
       auto& R = V->pr[i];
-      Limbs inv = H::inv_mod_2k(R.P2, sp);  // N^-1 mod R
-      Limbs np = H::resized(inv, sp);        // N' = R - N^-1 = two's complement of N^-1 mod R
+      Limbs np = H::resized(H::inv_mod_2k(R.P2, sp), sp);  // N' = R - N^-1 (two's complement)
       uint64_t cy = 1;
       for (auto& w : np) { cy += (uint32_t)~w; w = (uint32_t)cy; cy >>= 32; }
-      const std::vector<uint8_t> nb = bytes_of(R.P2, KB), npb = bytes_of(np, KB);
-      std::vector<uint8_t> b1((size_t)KB * KB, 0), b2h((size_t)KB * KB, 0), b2b((size_t)16 * KB, 0);
-      for (uint32_t n = 0; n < KB; n++)
-        for (uint32_t k = 0; k < KB; k++) {
-          if (k <= n) b1[flb::tc::cm_off(n, k, kch)] = npb[n - k];
-          const int64_t d = (int64_t)KB + n - k;
-          if (d >= 0 && d < (int64_t)KB) b2h[flb::tc::cm_off(n, k, kch)] = nb[d];
-        }
-      for (uint32_t j = 0; j < 16; j++)
-        for (uint32_t k = 0; k < KB; k++) {
-          const int64_t d = (int64_t)KB - 16 + j - k;
-          if (d >= 0 && d < (int64_t)KB) b2b[flb::tc::cm_off(j, k, kch)] = nb[d];
-        }
-      R.o_tcB1 = put_bytes(b1);
-      R.o_tcB2h = put_bytes(b2h);
-      R.o_tcB2b = put_bytes(b2b);
+      R.o_tcE1 = ext(bytes_of(np, KB), 2 * KB);
+      R.o_tcE2 = ext(bytes_of(R.P2, KB), 3 * KB);
     }
     V->tc = true;
   }

@@ -123,8 +123,8 @@ struct flb_priv {
     H::Schedule sched;
     size_t o_P, o_P2, o_R2, o_R3, o_Pinv, o_hR, o_sched;
     size_t o_nR;  // n R mod P^2 (key-holder encryption)
-    // tensor-core Montgomery operands for P^2 (flb_tc.cuh), core-matrix byte layout; 0 = absent
-    size_t o_tcB1 = 0, o_tcB2h = 0, o_tcB2b = 0;
+    // tensor-core Montgomery operands for P^2 (flb_tc.cuh): extended Toeplitz K-slices of N', N
+    size_t o_tcE1 = 0, o_tcE2 = 0;
   } pr[2];
   bool tc = false;  // tc operands present (sp in {32, 64})
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
@@ -502,13 +502,14 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
   static bool attr_done = false;
   if (!attr_done) {
     FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_pow<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_pow<S>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
     attr_done = true;
   }
   int sms = 0, dev_id = 0;
   FLB_CK(cudaGetDevice(&dev_id));
   FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id));
   const uint64_t tiles = (count + flb::tc::kTileM - 1) / flb::tc::kTileM;
-  const int grid = (int)std::min<uint64_t>((uint64_t)sms, tiles);
+  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), tiles);  // two CTAs per SM
   const int table = std::max(V->sched_p.table, V->sched_q.table);
   Scratch s_out, s_tab;
   int rc = s_out.alloc((size_t)2 * count * S * 4, st);
@@ -523,11 +524,11 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
     A.P2 = dev + R.o_P2;
     A.R2 = dev + R.o_R2;
     A.nR = dev + R.o_nR;
-    A.B1 = dev + R.o_tcB1;
-    A.B2h = dev + R.o_tcB2h;
-    A.B2b = dev + R.o_tcB2b;
+    A.E1 = dev + R.o_tcE1;
+    A.E2 = dev + R.o_tcE2;
     A.sched = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
     A.sched_len = (int)sc.ops.size();
+    if (A.sched_len < 2) return fail(FLB_EUNSUPPORTED, "tensor-core path needs a multi-window exponent");
     A.table = sc.table;
     A.y = y + (size_t)i * count * V->H;
     A.H = V->H;

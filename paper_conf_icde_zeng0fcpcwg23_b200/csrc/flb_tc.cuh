@@ -11,16 +11,22 @@
 // limb products, half of CIOS's 2 S^2) stays on the integer pipe.  The result is the canonical
 // Montgomery product, bit-identical to mont_mul (flb_bn.cuh).
 //
-// Tile: 128 elements per CTA (one per TMEM lane / MMA row), 512 threads.  Per multiplication:
-//   P   all 16 warps: groups of T = 4 lanes compute t = a b (row-scanning product, X = S/4 limbs
-//       per lane); t_lo goes to the MMA operand tile sA as bytes, t_hi to the element's work row;
-//   M1  one thread: D1[128 x 4S] = sA x B1 (B1[n][k] = N'_(n-k) bytes, n, k < 4S);
-//   N1  warps 0-3 (thread i = element i = TMEM lane i): carry-normalise D1's row into q mod R,
-//       written over sA;
-//   M2  one thread: D2 = sA x B2 for output byte columns 4S-16 .. 8S-1 (B2 = Toeplitz of N bytes);
-//   F   warps 0-3: u = t_hi + high(q N) + c', where the carry c' out of the low half is exact from
-//       the top 16 low columns alone (t_lo + (q N mod R) is a multiple of R; see stage F in tc_mont), then
-//       one conditional subtraction (u < 2N); u is written to the element's work row.
+// Tile: 128 elements per CTA (MMA M = 128, one per TMEM lane), 256 threads, two CTAs per SM so the
+// warp schedulers overlap one CTA's product phase (integer pipe) with the other's normalisation
+// (ALU, TMEM loads, barriers).  Per multiplication (KB = 4S bytes per operand):
+//   P   two halves of 64 elements: groups of T = 4 lanes compute t = a b (row-scanning product,
+//       X = S/4 limbs per lane, the multiplier staged in the element's sA row); t_lo goes to sA as
+//       bytes (the MMA A operand), t_hi to the element's work row;
+//   M1  one thread: D1[128 x KB] = sA x B1, B1[n][k] = N'_(n-k) (bytes, k <= n);
+//   N1  8 warps (TMEM lane quadrant w % 4, column half w / 4): q = D1 mod R normalised into bytes
+//       over sA, the carry between the column halves resolved exactly through shared memory;
+//   M2  one thread: D2 = sA x B2 for the byte columns [KB-8, 2KB-8) of q N (one N = KB MMA);
+//   F   8 warps: u = t_hi + high(q N) + c' (c' from the 8 columns below KB, the 7 top columns of
+//       q N from the top 8 bytes of q and N on the CUDA cores), one conditional subtraction.
+// The Toeplitz operands are stored once per K-slice shape: for K-slice ks the B operand is the
+// row window starting at KB - 32 ks (B1) or 2KB - 8 - 32 ks (B2) of an extended [rows][32 bytes]
+// matrix Ext[r][kk] = V_(r - KB - kk), so B1 and B2 take 2KB x 32 and 3KB x 32 bytes of shared
+// memory instead of KB x KB each.
 #pragma once
 #include <cstdint>
 #include "flb_kernels.cuh"  // flb_bn.cuh + the group load/store helpers
@@ -29,30 +35,27 @@ namespace flb {
 namespace tc {
 
 constexpr int kTileM = 128;     // elements per CTA tile (MMA M, TMEM lanes)
-constexpr int kThreads = 512;   // 16 warps
+constexpr int kThreads = 256;   // 8 warps; two CTAs per SM
+constexpr int kHalf = 64;       // elements per product half-phase
 constexpr int kT = 4;           // lanes per element in the product phase
-constexpr int kBoundary = 16;   // low columns of q N read for the carry into the high half
 
 template <int S>
 struct Cfg {
   static constexpr int X = S / kT;                 // limbs per lane
   static constexpr int KB = 4 * S;                 // bytes of an S-word operand (MMA K and N)
   static constexpr int KCH = KB / 16;              // 16-byte chunks per operand row
-  static constexpr int LD = X + 4;                 // staged multiplier row (words)
-  static constexpr int W0 = S + 16 > kT * LD ? S + 16 : kT * LD;
-  static constexpr int WROW = ((W0 + 3) / 4) % 2 == 0 ? ((W0 + 3) / 4) * 4 + 4 : ((W0 + 3) / 4) * 4;  // /4 odd
-  static constexpr int TMEM_COLS = 2 * KB <= 256 ? 256 : 512;
-  static constexpr int D2H_COL = KB;               // TMEM column of the high half of q N
+  static constexpr int QW = S / 2, QC = KB / 2;    // words / byte columns per normalising thread
+  static constexpr int WROW = ((S + 4) / 4) % 2 == 1 ? S + 4 : S + 8;  // work row (words), /4 odd
+  static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB)
   // dynamic shared memory carve-up (bytes)
-  static constexpr int OFF_B1 = 0;
-  static constexpr int OFF_B2H = OFF_B1 + KB * KB;
-  static constexpr int OFF_B2B = OFF_B2H + KB * KB;
-  static constexpr int OFF_A = OFF_B2B + kBoundary * KB;
-  static constexpr int OFF_W = OFF_A + kTileM * KB;
-  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;  // carry exchange, 4 x uint4 per element
-  static constexpr int SMEM = OFF_X + kTileM * 4 * 16;
+  static constexpr int OFF_E1 = 0;                          // 2 KB rows x 32 bytes
+  static constexpr int OFF_E2 = OFF_E1 + 2 * KB * 32;       // 3 KB rows x 32 bytes
+  static constexpr int OFF_A = OFF_E2 + 3 * KB * 32;        // 128 x KB bytes (core matrices)
+  static constexpr int OFF_W = OFF_A + kTileM * KB;         // 128 work rows
+  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, 2 x uint4 per element
+  static constexpr int SMEM = OFF_X + kTileM * 2 * 16;
   static_assert(KB <= 256, "one MMA covers N <= 256 output columns");
-  static_assert(X % 4 == 0, "16-byte limb chunks");
+  static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -76,11 +79,13 @@ __device__ __forceinline__ uint32_t idesc_u8(int m, int n) {
   return (2u << 4) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
 }
 
-// D[tmem] (+)= A[128 x 32k..] x B[n x 32k..]^T over kch/2 K-slices of 32 bytes
-__device__ __forceinline__ void mma_u8(uint32_t tmem_d, uint32_t sa, uint32_t sb, uint32_t kch, uint32_t idesc) {
+// D[tmem] = sum over the K-slices ks of A[:, 32 ks ..] x B_ks^T, B_ks the 8-row-aligned window of the
+// extended operand starting at row r0 - 32 ks
+__device__ __forceinline__ void mma_toeplitz(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext, uint32_t r0,
+                                             uint32_t idesc) {
   for (uint32_t ks = 0; ks < kch / 2; ks++) {
     const uint64_t ad = smem_desc(sa + ks * 256u, kch * 128u);
-    const uint64_t bd = smem_desc(sb + ks * 256u, kch * 128u);
+    const uint64_t bd = smem_desc(ext + ((r0 - 32u * ks) >> 3) * 256u, 256u);
     const uint32_t acc = ks > 0 ? 1u : 0u;
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
                  "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
@@ -102,8 +107,8 @@ __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.a
 __device__ __forceinline__ void tc_before_sync() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_after_sync() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
-// 32 consecutive s32 columns of this thread's TMEM lane (warp w owns lanes 32w .. 32w+31)
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+// consecutive s32 columns of this thread's TMEM lane (warp w owns lanes 32 (w % 4) ..)
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* v) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
       "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
@@ -112,19 +117,22 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
         "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
         "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
       : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
-
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
       : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
         "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
       : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t* v) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
-// four byte-column sums (each < 2^25) as one 32-bit-word contribution, plus a carry and an addend
+// four byte-column sums (each < 2^25) as one 32-bit-word contribution
 __device__ __forceinline__ uint64_t word_of(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3) {
   return (uint64_t)c0 + ((uint64_t)c1 << 8) + ((uint64_t)c2 << 16) + ((uint64_t)c3 << 24);
 }
@@ -135,45 +143,84 @@ struct Smem {
   uint64_t* mbar;
 };
 
+// An operand of tc_mont per element of the tile: the element's work row (row = true), or element j
+// of an array at p + j * stride with `words` limbs (the rest zero; elements >= `valid` read zeros;
+// stride 0 = one constant for all).
+struct Src {
+  const uint32_t* p;
+  uint32_t stride, words, valid;
+  bool row;
+};
+__device__ __forceinline__ Src src_row() { return Src{nullptr, 0, 0, 0, true}; }
+__device__ __forceinline__ Src src_arr(const uint32_t* p, uint32_t stride, uint32_t words, uint32_t valid) {
+  return Src{p, stride, words, valid, false};
+}
+
 #ifndef FLB_TC_PROF
 #define FLB_TC_PROF 0
 #endif
 #if FLB_TC_PROF
 // per-phase cycle totals of thread 0 (P, M1 wait, N1, M2 wait, F, calls): FLB_TC_PROF=1 builds only
 static __device__ unsigned long long g_tc_prof[8];
-#define TC_MARK(slot)                                              \
-  do {                                                             \
-    if (threadIdx.x == 0) {                                        \
-      const long long now_ = clock64();                            \
+#define TC_MARK(slot)                                               \
+  do {                                                              \
+    if (threadIdx.x == 0) {                                         \
+      const long long now_ = clock64();                             \
       atomicAdd(&g_tc_prof[slot], (unsigned long long)(now_ - t_)); \
-      t_ = now_;                                                   \
-    }                                                              \
+      t_ = now_;                                                    \
+    }                                                               \
   } while (0)
 #else
 #define TC_MARK(slot) do {} while (0)
 #endif
 
-// Montgomery product of the tile: this group's element has a, b in registers (X limbs per lane);
-// on return the canonical a b R^-1 mod N is in the element's work row (words 0..S-1).  `phase`
-// tracks the mbarrier parity (two completions per call).  Collective over the whole CTA.
 template <int S>
-__device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const uint32_t (&b)[Cfg<S>::X],
-                                        const Smem& sm, const uint32_t* __restrict__ Nmod, uint32_t& phase) {
+__device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s, int elem, const uint32_t* sW) {
   using C = Cfg<S>;
-  constexpr int X = C::X, LD = C::LD, KCH = C::KCH, KB = C::KB;
-  const int tid = threadIdx.x, elem = tid / kT, k = tid % kT, warp = tid >> 5;
+  const int k = threadIdx.x % kT;
+  if (s.row) {
+    const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + k * C::X);
+#pragma unroll
+    for (int v = 0; v < C::X / 4; v++) {
+      const uint4 u = q[v];
+      r[4 * v] = u.x; r[4 * v + 1] = u.y; r[4 * v + 2] = u.z; r[4 * v + 3] = u.w;
+    }
+  } else {
+    load_elem<C::X, kT>(r, s.p + (size_t)elem * s.stride, s.words, (uint32_t)elem < s.valid);
+  }
+}
+
+// Montgomery product over the tile: for every element, a b R^-1 mod N (canonical) into its work
+// row.  sq: b = a.  `phase` tracks the mbarrier parity (two completions per call).  CTA-collective.
+template <int S>
+__device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, const Smem& sm,
+                                        const uint32_t* __restrict__ Nmod, uint32_t& phase) {
+  using C = Cfg<S>;
+  constexpr int X = C::X, KCH = C::KCH, KB = C::KB, QW = C::QW, QC = C::QC;
+  const int tid = threadIdx.x, k = tid % kT, warp = tid >> 5;
   uint8_t* sA = sm.base + C::OFF_A;
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
-  uint32_t* grp = sW + elem * C::WROW;
 #if FLB_TC_PROF
   long long t_ = clock64();
 #endif
-  // ---- P: t = a b (rows of b's words staged in the element's work row)
-  {
-    __syncwarp();
-    uint4* q = reinterpret_cast<uint4*>(grp + k * LD);
+  // ---- P: t = a b, two halves of 64 elements
+#pragma unroll 1
+  for (int h = 0; h < 2; h++) {
+    const int elem = h * kHalf + tid / kT;
+    uint32_t a[X], b[X];
+    src_load<S>(a, sa, elem, sW);
+    if (sq) {
 #pragma unroll
-    for (int v = 0; v < X / 4; v++) q[v] = make_uint4(b[4 * v], b[4 * v + 1], b[4 * v + 2], b[4 * v + 3]);
+      for (int j = 0; j < X; j++) b[j] = a[j];
+    } else {
+      src_load<S>(b, sb, elem, sW);
+    }
+    // stage b in the element's sA row (natural byte order: word w at chunk w / 4)
+    __syncwarp();
+#pragma unroll
+    for (int v = 0; v < X / 4; v++)
+      *reinterpret_cast<uint4*>(sA + cm_off(elem, 16u * (k * X / 4 + v), KCH)) =
+          make_uint4(b[4 * v], b[4 * v + 1], b[4 * v + 2], b[4 * v + 3]);
     __syncwarp();
     uint32_t E[X + 1], O[X + 1], pend = 0, lo[X], hi[X];
     const uint32_t dummy[X] = {};
@@ -183,11 +230,15 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
     for (int t = 0; t < X; t++) lo[t] = 0;
 #pragma unroll 1
     for (int kk = 0; kk < kT; kk++) {
-      const uint32_t* row = grp + kk * LD;
 #pragma unroll
-      for (int jj = 0; jj < X; jj++) {
-        const uint32_t w = cios_step<X, kT, false>(E, O, pend, a, row[jj], dummy, 0u);
-        if (k == kk) lo[jj] = w;
+      for (int j4 = 0; j4 < X; j4 += 4) {
+        const uint4 bq = *reinterpret_cast<const uint4*>(sA + cm_off(elem, 4u * (kk * X + j4), KCH));
+        const uint32_t bw[4] = {bq.x, bq.y, bq.z, bq.w};
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          const uint32_t o = cios_step<X, kT, false>(E, O, pend, a, bw[u], dummy, 0u);
+          if (k == kk) lo[j4 + u] = o;
+        }
       }
     }
     collapse<X, kT>(hi, E, O, pend);
@@ -196,44 +247,32 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
     for (int v = 0; v < X / 4; v++) {
       *reinterpret_cast<uint4*>(sA + cm_off(elem, 16u * (k * X / 4 + v), KCH)) =
           make_uint4(lo[4 * v], lo[4 * v + 1], lo[4 * v + 2], lo[4 * v + 3]);
-      *reinterpret_cast<uint4*>(grp + k * X + 4 * v) = make_uint4(hi[4 * v], hi[4 * v + 1], hi[4 * v + 2], hi[4 * v + 3]);
+      *reinterpret_cast<uint4*>(sW + elem * C::WROW + k * X + 4 * v) =
+          make_uint4(hi[4 * v], hi[4 * v + 1], hi[4 * v + 2], hi[4 * v + 3]);
     }
-    fence_async_smem();
   }
+  fence_async_smem();
   tc_before_sync();
   __syncthreads();
   TC_MARK(0);
-  // ---- M1: q columns
+  // ---- M1: q columns [0, KB)
   if (tid == 0) {
     tc_after_sync();
-    mma_u8(sm.tmem, smem_u32(sA), smem_u32(sm.base + C::OFF_B1), KCH, idesc_u8(kTileM, KB));
+    mma_toeplitz(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E1), KB, idesc_u8(kTileM, KB));
     mma_commit(sm.mbar);
   }
-  // every warp normalises: TMEM lane quadrant L = warp % 4 (elements 32L .. 32L+31), column quarter
-  // g = warp / 4 (QW words = QC byte columns); carries cross quarters through `xch` (exact)
-  constexpr int QW = S / 4, QC = 4 * QW;
+  // normalisation: TMEM lane quadrant L = warp % 4 (elements 32L ..), column half g = warp / 4
   const int L = warp & 3, g = warp >> 2, i = 32 * L + (tid & 31);
   const uint32_t lane_base = sm.tmem + ((uint32_t)(32 * L) << 16);
   uint32_t* row = sW + i * C::WROW;
-  uint4* xch = reinterpret_cast<uint4*>(sm.base + C::OFF_X) + i * 4;
-  uint4 ttop = make_uint4(0, 0, 0, 0);
-  if (g == 0) ttop = *reinterpret_cast<const uint4*>(sA + cm_off(i, KB - 16, KCH));  // t_lo top 16 bytes
+  uint4* xch = reinterpret_cast<uint4*>(sm.base + C::OFF_X) + i * 2;
+  uint2 ttop = make_uint2(0, 0);
+  if (g == 0) ttop = *reinterpret_cast<const uint2*>(sA + cm_off(i, KB - 8, KCH));  // t_lo bytes KB-8 ..
   mbar_wait(sm.mbar, phase);
   phase ^= 1u;
   tc_after_sync();
   TC_MARK(1);
   uint32_t v[QW];
-  // carry into this quarter from the quarters below: cin_{h+1} = C_h + [word0_h + cin_h overflows
-  // and words 1.. of quarter h are all ones]; returns the carry out of quarter `upto` - 1
-  auto resolve = [&](int upto) {
-    uint64_t cin = 0;
-    for (int h = 0; h < upto; h++) {
-      const uint4 x = xch[h];
-      const uint64_t ov = (x.z != 0u && (((uint64_t)x.y + cin) >> 32) != 0) ? 1u : 0u;
-      cin = (uint64_t)x.x + ov;
-    }
-    return cin;
-  };
   auto add_in = [&](uint64_t cin) {
 #pragma unroll
     for (int w = 0; w < QW; w++) {
@@ -242,13 +281,26 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
       cin = s >> 32;
     }
   };
-  // ---- N1: q = D1 mod R (quarter g, local carry chain), bytes back into sA
+  auto publish = [&](uint64_t carry) {
+    uint32_t ao = 0xffffffffu;
+#pragma unroll
+    for (int w = 1; w < QW; w++) ao &= v[w];
+    xch[g] = make_uint4((uint32_t)carry, v[0], ao == 0xffffffffu ? 1u : 0u, 0u);
+  };
+  // carry into half 1 (= out of half 0), and out of half 1
+  auto carry_out = [&](int h, uint64_t cin) {
+    const uint4 x = xch[h];
+    const uint64_t ov = (x.z != 0u && (((uint64_t)x.y + cin) >> 32) != 0) ? 1u : 0u;
+    return (uint64_t)x.x + ov;
+  };
+  // ---- N1: q = D1 mod R
   {
     uint64_t carry = 0;
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
       uint32_t cv[32];
       tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
+      tmem_wait();
 #pragma unroll
       for (int w = 0; w < 8; w++) {
         const uint64_t s = carry + word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]);
@@ -256,25 +308,21 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
         carry = s >> 32;
       }
     }
-    uint32_t ao = 0xffffffffu;
-#pragma unroll
-    for (int w = 1; w < QW; w++) ao &= v[w];
-    xch[g] = make_uint4((uint32_t)carry, v[0], ao == 0xffffffffu ? 1u : 0u, 0u);
+    publish(carry);
   }
   tc_before_sync();
-  __syncthreads();  // all D1 reads and all t_lo reads of sA done; carries published
-  add_in(resolve(g));
+  __syncthreads();  // D1 drained, t_lo bytes read, carries published
+  if (g == 1) add_in(carry_out(0, 0));
 #pragma unroll
   for (int c = 0; c < QW / 4; c++)
     *reinterpret_cast<uint4*>(sA + cm_off(i, g * QC + 16 * c, KCH)) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
   fence_async_smem();
   tc_before_sync();
   __syncthreads();
-  // ---- M2: q N, columns 4S-16 .. 8S-1
+  // ---- M2: q N columns [KB-8, 2KB-8) into D2 = TMEM [0, KB)
   if (tid == 0) {
     tc_after_sync();
-    mma_u8(sm.tmem + C::D2H_COL, smem_u32(sA), smem_u32(sm.base + C::OFF_B2H), KCH, idesc_u8(kTileM, KB));
-    mma_u8(sm.tmem, smem_u32(sA), smem_u32(sm.base + C::OFF_B2B), KCH, idesc_u8(kTileM, kBoundary));
+    mma_toeplitz(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E2), 2 * KB - 8, idesc_u8(kTileM, KB));
     mma_commit(sm.mbar);
   }
   TC_MARK(2);
@@ -282,29 +330,57 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
   phase ^= 1u;
   tc_after_sync();
   TC_MARK(3);
-  // ---- F: u = t_hi + high(q N) + c'.  The carry out of the low half: t_lo + (q N mod R) = c' R
-  // exactly; with W = the top 16 low byte columns of t + q N (as an integer over those columns) and
-  // Z the rest (< 2^(8(4S-16)+26)), c' R = W 2^(8(4S-16)) + Z, so c' = ceil(W / 2^128): the floor
-  // plus one when W mod 2^128 != 0.  Quarter 0 starts its chain with c'.
+  // ---- F: u = t_hi + high(q N) + c'.  t_lo + (q N mod R) = c' R exactly; with W = the 8 byte
+  // columns below KB of t + q N (as an integer over those columns) and Z the rest
+  // (< 2^(8(KB-8)+26)), c' R = W 2^(8(KB-8)) + Z, so c' = ceil(W / 2^64).  Half 0 starts with c'.
   {
     uint64_t carry = 0;
     if (g == 0) {
-      uint32_t bc[16];
-      tmem_ld16(lane_base, bc);
-      const uint32_t tt[4] = {ttop.x, ttop.y, ttop.z, ttop.w};
-      uint32_t nz = 0;
+      uint32_t bc[8];
+      tmem_ld8(lane_base, bc);
+      tmem_wait();
+      const uint64_t s0 = word_of(bc[0], bc[1], bc[2], bc[3]) + ttop.x;
+      const uint64_t s1 = (s0 >> 32) + word_of(bc[4], bc[5], bc[6], bc[7]) + ttop.y;
+      carry = (s1 >> 32) + ((((uint32_t)s0) | ((uint32_t)s1)) != 0u ? 1u : 0u);
+    }
+    // this half's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; half 1's last 8 columns
+    // (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
+    uint32_t top[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    if (g == 1) {
+      const uint2 qt2 = *reinterpret_cast<const uint2*>(sA + cm_off(i, KB - 8, KCH));
+      const uint2 nt2 = __ldg(reinterpret_cast<const uint2*>(Nmod + S - 2));
+      uint32_t qt[8], nt[8];
 #pragma unroll
-      for (int w = 0; w < 4; w++) {
-        const uint64_t s = carry + word_of(bc[4 * w], bc[4 * w + 1], bc[4 * w + 2], bc[4 * w + 3]) + tt[w];
-        nz |= (uint32_t)s;
-        carry = s >> 32;
+      for (int b = 0; b < 4; b++) {
+        qt[b] = (qt2.x >> (8 * b)) & 0xffu; qt[4 + b] = (qt2.y >> (8 * b)) & 0xffu;
+        nt[b] = (nt2.x >> (8 * b)) & 0xffu; nt[4 + b] = (nt2.y >> (8 * b)) & 0xffu;
       }
-      carry += nz != 0u ? 1u : 0u;
+#pragma unroll
+      for (int j = 0; j < 7; j++) {
+        uint32_t acc = 0;
+#pragma unroll
+        for (int a2 = j + 1; a2 < 8; a2++) acc += qt[a2] * nt[j - a2 + 8];
+        top[j] = acc;
+      }
     }
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
       uint32_t cv[32];
-      tmem_ld32(lane_base + (uint32_t)(C::D2H_COL + g * QC + c0), cv);
+      const uint32_t col = 8u + (uint32_t)(g * QC + c0);
+      if (c0 + 32 < QC) {
+        tmem_ld32(lane_base + col, cv);
+      } else {
+        // last chunk of the half: D2 columns col .. col+23 always exist; col+24 .. col+31 exist
+        // for half 0 only (half 1's are the top columns)
+        tmem_ld16(lane_base + col, cv);
+        tmem_ld8(lane_base + col + 16u, cv + 16);
+        uint32_t t8[8];
+        tmem_ld8(lane_base + (g == 0 ? col + 24u : 0u), t8);  // uniform per warp; unused for half 1
+        tmem_wait();
+#pragma unroll
+        for (int j = 0; j < 8; j++) cv[24 + j] = g == 0 ? t8[j] : top[j];
+      }
+      tmem_wait();
       const uint4 h0 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[0];
       const uint4 h1 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[1];
       const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
@@ -315,16 +391,14 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
         carry = s >> 32;
       }
     }
-    uint32_t ao = 0xffffffffu;
-#pragma unroll
-    for (int w = 1; w < QW; w++) ao &= v[w];
-    xch[g] = make_uint4((uint32_t)carry, v[0], ao == 0xffffffffu ? 1u : 0u, 0u);
+    publish(carry);
   }
   tc_before_sync();
   __syncthreads();
-  const uint64_t ovf = resolve(4);  // bit above S words (u < 2N < 2R)
-  add_in(resolve(g));
-  // u - N over this quarter: local borrow B_g, zero-difference flag Z_g
+  const uint64_t c1 = carry_out(0, 0);
+  const uint64_t ovf = carry_out(1, c1);  // bit above S words (u < 2N < 2R)
+  if (g == 1) add_in(c1);
+  // u - N over this half: local borrow and zero-difference flag
   uint32_t d[QW];
   {
     uint32_t br = 0, nzd = 0;
@@ -344,15 +418,11 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
   }
   __syncthreads();
   {
-    uint32_t bin = 0, bout;
-    for (int h = 0; h < 4; h++) {
-      if (h == g) bout = bin;  // borrow into this quarter
-      const uint32_t f = xch[h].w;
-      bin = (f & 1u) | ((f >> 1) & bin);
-    }
-    const bool take = ovf != 0 || bin == 0;  // u >= N
-    if (take) {
-      uint32_t br = bout;
+    const uint32_t f0 = xch[0].w, f1 = xch[1].w;
+    const uint32_t b1 = f0 & 1u;                          // borrow into half 1
+    const uint32_t bout = (f1 & 1u) | ((f1 >> 1) & b1);    // borrow out of the top
+    if (ovf != 0 || bout == 0) {                           // u >= N: take u - N
+      uint32_t br = g == 1 ? b1 : 0u;
 #pragma unroll
       for (int w = 0; w < QW; w++) {
         const uint64_t df = (uint64_t)d[w] - br;
@@ -372,24 +442,45 @@ __device__ __forceinline__ void tc_mont(const uint32_t (&a)[Cfg<S>::X], const ui
 #endif
 }
 
-// this group's X limbs of the element's work row
+// copy each element's work row (words 0..S-1) to dst + j * stride (elements j < valid)
 template <int S>
-__device__ __forceinline__ void tc_row_load(uint32_t (&r)[Cfg<S>::X], const Smem& sm) {
+__device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint32_t stride, uint32_t valid) {
   using C = Cfg<S>;
-  const int elem = threadIdx.x / kT, k = threadIdx.x % kT;
-  const uint32_t* row = reinterpret_cast<const uint32_t*>(sm.base + C::OFF_W) + elem * C::WROW + k * C::X;
+  const uint32_t* sW = reinterpret_cast<const uint32_t*>(sm.base + C::OFF_W);
+  const int k = threadIdx.x % kT;
+#pragma unroll 1
+  for (int h = 0; h < 2; h++) {
+    const int elem = h * kHalf + threadIdx.x / kT;
+    if ((uint32_t)elem < valid) {
+      const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + k * C::X);
+      uint4* o = reinterpret_cast<uint4*>(dst + (size_t)elem * stride + k * C::X);
 #pragma unroll
-  for (int v = 0; v < C::X / 4; v++) {
-    const uint4 u = reinterpret_cast<const uint4*>(row)[v];
-    r[4 * v] = u.x; r[4 * v + 1] = u.y; r[4 * v + 2] = u.z; r[4 * v + 3] = u.w;
+      for (int v = 0; v < C::X / 4; v++) o[v] = q[v];
+    }
   }
 }
 
-}  // namespace tc
-}  // namespace flb
-
-namespace flb {
-namespace tc {
+// work row <- (row + 1) mod N for every element (row < N)
+template <int S>
+__device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* __restrict__ Nmod) {
+  using C = Cfg<S>;
+  constexpr int X = C::X;
+  uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
+  const int k = threadIdx.x % kT;
+#pragma unroll 1
+  for (int h = 0; h < 2; h++) {
+    const int elem = h * kHalf + threadIdx.x / kT;
+    uint32_t r[X], nn[X];
+    src_load<S>(r, src_row(), elem, sW);
+    load_const<X, kT>(nn, Nmod);
+    grp_add_small<X, kT>(r, 1u);
+    grp_cond_sub<X, kT>(r, nn, 0u);
+    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + k * X);
+#pragma unroll
+    for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
+  }
+  __syncthreads();
+}
 
 // ----------------------------------------------------------------------------- key-holder stage 2
 // c_P = (1 + m n) y^P mod P^2 for one prime P per launch (Eq. 3 with g = n + 1, by the
@@ -400,10 +491,9 @@ struct PowArgs {
   const uint32_t* P2;      // modulus P^2 (S words)
   const uint32_t* R2;      // R^2 mod P^2
   const uint32_t* nR;      // n R mod P^2
-  const uint32_t* B1;      // Toeplitz(N') core-matrix operand, KB x KB bytes
-  const uint32_t* B2h;     // Toeplitz(N) high columns, KB x KB bytes
-  const uint32_t* B2b;     // Toeplitz(N) boundary columns, 16 x KB bytes
-  const uint32_t* sched;   // schedule of the exponent P
+  const uint32_t* E1;      // extended Toeplitz(N') operand, 2KB x 32 bytes (core matrices)
+  const uint32_t* E2;      // extended Toeplitz(N) operand, 3KB x 32 bytes
+  const uint32_t* sched;   // schedule of the exponent P (at least one op after the first window)
   int sched_len, table;
   const uint32_t* y;       // [count][H]
   uint32_t H;
@@ -414,22 +504,20 @@ struct PowArgs {
 };
 
 template <int S>
-__global__ void __launch_bounds__(kThreads, 1) k_tc_pow(const PowArgs A) {
+__global__ void __launch_bounds__(kThreads, 2) k_tc_pow(const PowArgs A) {
   using C = Cfg<S>;
-  constexpr int X = C::X, KB = C::KB;
+  constexpr int KB = C::KB;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t tmem_sh;
-  const int tid = threadIdx.x, warp = tid >> 5, elem = tid / kT, k = tid % kT;
+  const int tid = threadIdx.x, warp = tid >> 5;
   {
-    const uint4* s1 = reinterpret_cast<const uint4*>(A.B1);
-    const uint4* s2 = reinterpret_cast<const uint4*>(A.B2h);
-    const uint4* s3 = reinterpret_cast<const uint4*>(A.B2b);
-    uint4* d1 = reinterpret_cast<uint4*>(smem + C::OFF_B1);
-    uint4* d2 = reinterpret_cast<uint4*>(smem + C::OFF_B2H);
-    uint4* d3 = reinterpret_cast<uint4*>(smem + C::OFF_B2B);
-    for (int i = tid; i < KB * KB / 16; i += kThreads) { d1[i] = __ldg(s1 + i); d2[i] = __ldg(s2 + i); }
-    for (int i = tid; i < kBoundary * KB / 16; i += kThreads) d3[i] = __ldg(s3 + i);
+    const uint4* s1 = reinterpret_cast<const uint4*>(A.E1);
+    const uint4* s2 = reinterpret_cast<const uint4*>(A.E2);
+    uint4* d1 = reinterpret_cast<uint4*>(smem + C::OFF_E1);
+    uint4* d2 = reinterpret_cast<uint4*>(smem + C::OFF_E2);
+    for (int i = tid; i < 2 * KB * 32 / 16; i += kThreads) d1[i] = __ldg(s1 + i);
+    for (int i = tid; i < 3 * KB * 32 / 16; i += kThreads) d2[i] = __ldg(s2 + i);
   }
   if (tid == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&mbar)));
@@ -448,59 +536,45 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_pow(const PowArgs A) {
   uint32_t phase = 0;
   const int TB = A.table;
   uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * (TB + 1) * S;
-  auto slot = [&](int ent) { return tab + ((size_t)ent * kTileM + elem) * S + k * X; };
+  auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
+  auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
+  const Src row = src_row();
   for (uint64_t tile = blockIdx.x; tile * kTileM < A.count; tile += gridDim.x) {
-    const uint64_t e = tile * kTileM + elem;
-    const bool valid = e < A.count;
-    uint32_t a[X], b[X];
-    load_elem<X, kT>(a, A.y + e * A.H, A.H, valid);
-    load_const<X, kT>(b, A.R2);
-    tc_mont<S>(a, b, sm, A.P2, phase);                     // x = y R mod P^2
-    tc_row_load<S>(a, sm);
-    store_limbs<X>(slot(0), a);
+    const uint64_t e0 = tile * kTileM;
+    const uint32_t nvalid = (uint32_t)((A.count - e0) < (uint64_t)kTileM ? (A.count - e0) : (uint64_t)kTileM);
+    tc_mont<S>(src_arr(A.y + e0 * A.H, A.H, A.H, nvalid), src_arr(A.R2, 0, S, kTileM), false, sm, A.P2, phase);
+    tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x = y R mod P^2
     if (TB > 1) {
-      tc_mont<S>(a, a, sm, A.P2, phase);                   // x^2
-      tc_row_load<S>(b, sm);
+      tc_mont<S>(row, row, true, sm, A.P2, phase);            // x^2
+      tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
 #pragma unroll 1
-      for (int i = 1; i < TB; i++) {
-        load_limbs_plain<X>(a, slot(i - 1));
-        tc_mont<S>(a, b, sm, A.P2, phase);
-        tc_row_load<S>(a, sm);
-        store_limbs<X>(slot(i), a);
+      for (int t = 1; t < TB; t++) {
+        tc_mont<S>(slot(t - 1), slot(TB), false, sm, A.P2, phase);
+        tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
       }
     }
     const uint32_t op0 = __ldg(A.sched);
-    load_limbs_plain<X>(a, slot((int)(op0 >> 16) - 1));
+    Src cur = slot((int)(op0 >> 16) - 1);
 #pragma unroll 1
     for (int o = 1; o < A.sched_len; o++) {
       const uint32_t op = __ldg(A.sched + o);
       const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
 #pragma unroll 1
-      for (int i = 0; i < sq; i++) {
-        tc_mont<S>(a, a, sm, A.P2, phase);
-        tc_row_load<S>(a, sm);
+      for (int t = 0; t < sq; t++) {
+        tc_mont<S>(cur, cur, true, sm, A.P2, phase);
+        cur = row;
       }
       if (idx >= 0) {
-        load_limbs_plain<X>(b, slot(idx));
-        tc_mont<S>(a, b, sm, A.P2, phase);
-        tc_row_load<S>(a, sm);
+        tc_mont<S>(cur, slot(idx), false, sm, A.P2, phase);
+        cur = row;
       }
     }
-    store_limbs<X>(slot(TB), a);                           // y^P R
-    load_elem<X, kT>(a, A.m + e * S, S, valid);
-    load_const<X, kT>(b, A.nR);
-    tc_mont<S>(a, b, sm, A.P2, phase);                     // m n mod P^2
-    tc_row_load<S>(b, sm);
-    {
-      uint32_t nn[X];
-      load_const<X, kT>(nn, A.P2);
-      grp_add_small<X, kT>(b, 1u);
-      grp_cond_sub<X, kT>(b, nn, 0u);                      // 1 + m n mod P^2
-    }
-    load_limbs_plain<X>(a, slot(TB));
-    tc_mont<S>(a, b, sm, A.P2, phase);                     // c_P
-    tc_row_load<S>(a, sm);
-    if (valid) store_limbs<X>(A.out + e * S + k * X, a);
+    tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);             // y^P R
+    tc_mont<S>(src_arr(A.m + e0 * S, S, S, nvalid), src_arr(A.nR, 0, S, kTileM), false, sm, A.P2, phase);  // m n
+    tc_row_add_one<S>(sm, A.P2);                              // 1 + m n mod P^2
+    tc_mont<S>(slot(TB), row, false, sm, A.P2, phase);        // c_P
+    tc_row_store<S>(sm, A.out + e0 * S, S, nvalid);
+    __syncthreads();  // the work rows are rewritten by the next tile's first product
   }
   tc_before_sync();
   __syncthreads();
