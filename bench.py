@@ -369,21 +369,57 @@ def run_flb(args):
     other_rate = ops_enc / world / (e0.elapsed_time(e1) * 1e-3)
 
     # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
+    tc_on = os.environ.get("FLB_TC", "1") != "0"
+    enc_tc = dec_tc = None
+    if tc_on:
+        try:
+            enc_tc = flb.op_cost(priv, "encrypt_crt_tc")
+            dec_tc = flb.op_cost(priv, "decrypt_tc")
+        except flb.FlbError:
+            enc_tc = dec_tc = None
     if args.encrypt == "keyholder":
         enc_mm, enc_lp = flb.op_cost(priv, "encrypt_crt")
-        enc_kernel = ("k_encrypt_crt<16,4>" if os.environ.get("FLB_CRT_V1") == "1"
-                      else "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)")
+        if enc_tc:
+            enc_kernel = ("k_tc_exp<32> + k_tc_exp<64> (two-stage key-holder encryption; Montgomery reduction as "
+                          "u8 tcgen05 MMAs, t = a b on the IMAD pipe)")
+        else:
+            enc_kernel = ("k_encrypt_crt<16,4>" if os.environ.get("FLB_CRT_V1") == "1"
+                          else "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)")
     else:
         enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
         enc_kernel = "k_encrypt<16,8>"
+        enc_tc = None
     dec_mm, dec_lp = flb.op_cost(priv, "decrypt")
-    enc_lp_launch = enc_lp * CLIENTS * rows
-    achieved = enc_lp_launch / (phase["t_enc"] * 1e-3) / 1e12
+    enc_units = CLIENTS * rows
     sm_mhz_max = clk.get("sm_max_mhz") or 1965.0
     peak = 148 * PEAK_LP_PER_CLK_SM * sm_mhz_max * 1e6 / 1e12
+    # u8 MMA peak: tools/tc_i8_probe.cu measured 7.26K MAC/clk/SM (kind::i8, M=128 N=256)
+    mma_peak = 148 * 7260 * sm_mhz_max * 1e6 / 1e12
+    if enc_tc:
+        # IMAD-pipe work the tensor-core kernels actually issue: S^2 per Montgomery product
+        imad_lp = enc_tc[1]
+        achieved = imad_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12
+        per_unit = {"mont_muls": enc_tc[0], "imad_limb_products": imad_lp, "u8_macs": 32 * imad_lp,
+                    "cios_equivalent_limb_products": enc_lp}
+        tensor = {"achieved": 32 * imad_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12, "peak": mma_peak,
+                  "unit": "T u8 MAC/s (tcgen05.mma kind::i8)",
+                  "peak_basis": "148 SM x 7.26K MAC/clk/SM (tools/tc_i8_probe.cu) x %.0f MHz" % sm_mhz_max}
+        tensor["frac"] = tensor["achieved"] / mma_peak
+        cios_eq = enc_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12
+    else:
+        achieved = enc_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12
+        per_unit = {"mont_muls": enc_mm, "limb_products": enc_lp}
+        tensor = None
+        cios_eq = achieved
+    dec_roof = None
+    if dec_tc:
+        dec_roof = {"kernel": "k_tc_exp<64> + k_dec_finish<16,4>", "mont_muls_tc": dec_tc[0],
+                    "imad_limb_products": dec_tc[1],
+                    "imad_achieved": dec_tc[1] * rows / (phase["t_dec"] * 1e-3) / 1e12,
+                    "frac": dec_tc[1] * rows / (phase["t_dec"] * 1e-3) / 1e12 / peak}
     traffic = None
     tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json" if args.encrypt == "public" else
-                      "encrypt_crt_traffic.json")
+                      ("encrypt_tc_traffic.json" if enc_tc else "encrypt_crt_traffic.json"))
     if os.path.exists(tp):
         try:
             with open(tp) as f:
@@ -456,7 +492,12 @@ def run_flb(args):
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": r["sample"],
                "per_op_seconds": {"encrypt": r["t_enc"], "decrypt": r["t_dec"], "add": r["t_add"]}}
 
-    launches_per_step = CLIENTS + 1 + 3 + (3 if world > 1 else 0) + 1 + (1 if my_values else 0)
+    # pack per client; encrypt (TC: Philox fill, k_tc_exp<32>, k_tc_exp<64>, k_crt_combine; CIOS:
+    # k_crt_pre, k_encrypt_crt2); reduce (plan scan, plan fill, k_reduce); exchange + finish (N > 1);
+    # decrypt (TC: k_tc_exp<64>, k_dec_finish; CIOS: k_decrypt); unpack
+    enc_launches = (4 if enc_tc else 2) if args.encrypt == "keyholder" else 1
+    launches_per_step = (CLIENTS + enc_launches + 3 + (3 if world > 1 else 0) + (2 if dec_tc else 1)
+                         + (1 if my_values else 0))
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -479,11 +520,12 @@ def run_flb(args):
             "encrypt_mode": args.encrypt,
             "roofline": {"bound": "alu", "kernel": enc_kernel, "achieved": achieved, "peak": peak,
                          "unit": "T limb-products/s (IMAD.WIDE.U32 32x32->64, FMA-heavy pipe)",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "per_unit": {"mont_muls": enc_mm, "limb_products": enc_lp},
+                         "frac": achieved / peak, "traffic": traffic, "per_unit": per_unit,
                          "peak_basis": "148 SM x 32 IMAD.WIDE/clk/SM x %.0f MHz (guide: IMAD rt=2/SMSP; "
-                                       "IMAD.WIDE half rate, measured tools/imad_peak.cu)" % sm_mhz_max},
+                                       "IMAD.WIDE half rate, measured tools/imad_peak.cu)" % sm_mhz_max,
+                         "tensor": tensor, "cios_equivalent_achieved": cios_eq},
             "decrypt_cost": {"mont_muls": dec_mm, "limb_products": dec_lp},
+            "decrypt_roofline": dec_roof,
             "clocks": clk, "gpu_launches": launches_per_step * args.steps,
             "e2e": e2e, "cpu_baseline": cpu,
         }

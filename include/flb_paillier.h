@@ -93,12 +93,20 @@ int flb_encrypt(const flb_pub* pub, const uint32_t* m, const uint32_t* r, uint64
  * ctr0 -> the same bits), computed as (1 + m n) r^n mod p^2 and mod q^2 with half-size moduli and
  * recombined by CRT (c = c_q + q^2 ((c_p - c_q) (q^2)^-1 mod p^2)) — about half the limb products.
  * Beyond the paper; in Fig. 2 the clients that encrypt also
- * decrypt, so they hold the key.  Arguments and errors as flb_encrypt. */
+ * decrypt, so they hold the key.  From 2048 bits the exponentiation is two-stage,
+ * r^n mod P^2 = (r^Q mod P)^P mod P^2; for 1024/2048-bit keys (P^2 of 32/64 words) and the
+ * half-frame first stage at 2048-4096 bits every Montgomery product runs its reduction
+ * q = t N' mod R, (t + q N)/R as u8 tcgen05 MMAs against Toeplitz matrices of N' and N (the batch
+ * shares N) with TMEM accumulators (csrc/flb_tc.cuh); FLB_TC=0 in the environment selects the
+ * CUDA-core CIOS kernels (same bits).  Scratch: stream-ordered, about 2 count (ct_words) words.
+ * Arguments and errors as flb_encrypt. */
 int flb_encrypt_crt(const flb_priv* priv, const uint32_t* m, const uint32_t* r, uint64_t seed,
                     uint64_t ctr0, uint32_t* c, size_t count, void* stream);
 
 /* Paillier::decrypt (Eq. 4), by CRT (reading c10).  c: [count][ct_words]
- * (each a unit < n^2), m: [count][pt_words] receives m_i in [0, n).  Errors: FLB_EINVAL, FLB_ECUDA. */
+ * (each a unit < n^2), m: [count][pt_words] receives m_i in [0, n).  For 1024/2048-bit keys the two
+ * exponentiations c^(P-1) mod P^2 run on the tensor-core Montgomery kernel (see flb_encrypt_crt;
+ * FLB_TC=0 selects CIOS, same bits).  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_decrypt(const flb_priv* priv, const uint32_t* c, uint32_t* m, size_t count, void* stream);
 
 /* Paillier::add (Eq. 5): out_i = c1_i * c2_i mod n^2.  All
@@ -251,13 +259,24 @@ int flb_reduce_segments_host(const flb_pub* pub, const uint32_t* c_host, size_t 
 int flb_debug_mont_mul(const flb_pub* pub, const uint32_t* a, const uint32_t* b, uint32_t* out,
                        size_t count, void* stream);
 
+/* Debug: the plain product phase of the tensor-core Montgomery kernel (csrc/flb_tc.cuh): t_i = a_i b_i
+ * (square != 0: a_i^2, b ignored but must be valid) as 2 words-limb integers, for count <= 128
+ * elements of words in {32, 64} limbs.  a, b: [count][words], t: [count][2 words], device.
+ * Errors: FLB_EINVAL. */
+int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, uint32_t words,
+                         int square, void* stream);
+
 /* Algorithmic cost of one element of an op, for roofline accounting: *mont_muls = Montgomery
  * multiplications the kernel performs per element (window table, schedule, domain entry/exit),
  * *limb_products = their CIOS limb-product count (2s^2 + s per s-limb multiplication, s^2 for
  * the plain low-half product of the exact division).  op: 0 = encrypt (pub), 1 = decrypt
  * (priv), 2 = add (pub), 3 = one reduce input (pub; excludes the per-chunk fix-up),
- * 4 = key-holder encrypt (priv).
- * Host only.  Errors: FLB_EINVAL. */
+ * 4 = key-holder encrypt (priv); for the tensor-core kernels (k_tc_exp: Montgomery reduction as
+ * u8 MMAs, PAPER Alg. 1 L98-L114 restated as a contraction against the shared modulus), whose IMAD
+ * work is only the S^2 limb products of t = a b per S-word multiplication: 5 = key-holder encrypt
+ * (both stages, priv), 6 = decrypt's two exponentiations (priv); *limb_products = those S^2
+ * products (the u8 MACs are 32x that).
+ * Host only.  Errors: FLB_EINVAL; FLB_EUNSUPPORTED for ops 5/6 on keys without the path. */
 int flb_op_cost(const flb_pub* pub, const flb_priv* priv, int op, uint64_t* mont_muls,
                 uint64_t* limb_products);
 

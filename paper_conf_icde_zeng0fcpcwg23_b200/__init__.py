@@ -440,7 +440,8 @@ def reduce_segments_host(pub: PublicKey, c, offsets, idx=None, max_segment_len: 
     return out
 
 
-OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3, "encrypt_crt": 4}
+OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3, "encrypt_crt": 4, "encrypt_crt_tc": 5,
+       "decrypt_tc": 6}
 
 
 def op_cost(key, op: str) -> Tuple[int, int]:
@@ -450,6 +451,17 @@ def op_cost(key, op: str) -> Tuple[int, int]:
     priv = key.handle if isinstance(key, PrivateKey) else None
     check("flb_op_cost", LIB.flb_op_cost(pub, priv, OPS[op], ctypes.byref(mm), ctypes.byref(lp)))
     return mm.value, lp.value
+
+
+def debug_tc_product(a: torch.Tensor, b: torch.Tensor, square: bool = False, stream=None) -> torch.Tensor:
+    """The tensor-core Montgomery kernel's product phase alone: a_i b_i (or a_i^2) as 2w-limb rows,
+    w = a.shape[1] in {32, 64}, at most 128 rows (debugging and parity tests)."""
+    M = _check_batch(a, a.shape[1], "a")
+    _check_batch(b, a.shape[1], "b")
+    out = torch.empty((M, 2 * a.shape[1]), dtype=torch.int32, device=a.device)
+    check("flb_debug_tc_product", LIB.flb_debug_tc_product(_ptr(a), _ptr(b), _ptr(out), M, a.shape[1], int(square),
+                                                           _stream(stream)))
+    return out
 
 
 def debug_mont_mul(pub: PublicKey, a: torch.Tensor, b: torch.Tensor, out: Optional[torch.Tensor] = None,

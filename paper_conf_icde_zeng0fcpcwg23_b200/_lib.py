@@ -55,6 +55,7 @@ SIGNATURES = {
     "flb_unpack": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _U32, _P, _P]),
     "flb_unpack_sums": (ctypes.c_int, [_P, ctypes.POINTER(CodecStruct), _P, _SZ, _P, _P]),
     "flb_debug_mont_mul": (ctypes.c_int, [_P, _P, _P, _P, _SZ, _P]),
+    "flb_debug_tc_product": (ctypes.c_int, [_P, _P, _P, _U32, _U32, ctypes.c_int, _P]),
     "flb_mod_create": (ctypes.c_int, [_P, _U32, ctypes.POINTER(_P)]),
     "flb_mod_free": (None, [_P]),
     "flb_mod_words": (_U32, [_P]),

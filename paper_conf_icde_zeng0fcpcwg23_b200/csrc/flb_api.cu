@@ -111,18 +111,18 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
       V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
     }
   }
-  // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 frames of 1024- and 2048-bit keys:
-  // extended Toeplitz K-slices Ext[r][kk] = V_(r - KB - kk) (bytes, zero outside [0, KB)) of
-  // V = N' = -N^-1 mod R (2 KB rows) and V = N (3 KB rows), 32 bytes per row, in the K-major
-  // core-matrix layout the MMA descriptors describe
-  if ((sp == 32 || sp == 64) && V->H) {
-    const uint32_t KB = 4 * sp;
+  // tensor-core Montgomery operands (flb_tc.cuh): extended Toeplitz K-slices
+  // Ext[r][kk] = V_(r - KB - kk) (bytes, zero outside [0, KB)) of V = N' = -N^-1 mod R (2 KB rows)
+  // and V = N (3 KB rows), 32 bytes per row, in the K-major core-matrix layout the MMA descriptors
+  // describe; for the P^2 moduli when sp is 32 or 64 (decryption, key-holder encryption stage 2)
+  // and for the half-frame P moduli when H is 32 or 64 (key-holder encryption stage 1)
+  {
     auto bytes_of = [](const Limbs& v, size_t nbytes) {
       std::vector<uint8_t> b(nbytes, 0);
       for (size_t i = 0; i < nbytes && i / 4 < v.size(); i++) b[i] = (uint8_t)(v[i / 4] >> (8 * (i % 4)));
       return b;
     };
-    auto ext = [&](const std::vector<uint8_t>& vb, uint32_t rows) {
+    auto ext = [&](const std::vector<uint8_t>& vb, uint32_t KB, uint32_t rows) {
       std::vector<uint8_t> m((size_t)rows * 32, 0);
       for (uint32_t r = 0; r < rows; r++)
         for (uint32_t kk = 0; kk < 32; kk++) {
@@ -133,15 +133,27 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
       for (size_t i = 0; i < m.size(); i++) w[i / 4] |= (uint32_t)m[i] << (8 * (i % 4));
       return V->blob.put_raw(w);
     };
-    for (int i = 0; i < 2; i++) {
-      auto& R = V->pr[i];
-      Limbs np = H::resized(H::inv_mod_2k(R.P2, sp), sp);  // N' = R - N^-1 (two's complement)
+    // (E1, E2) offsets for modulus N in an S-word frame
+    auto operands = [&](const Limbs& N, uint32_t S, size_t* e1, size_t* e2) {
+      const uint32_t KB = 4 * S;
+      const Limbs Nf = H::resized(N, S);
+      Limbs np = H::resized(H::inv_mod_2k(Nf, S), S);  // N' = R - N^-1 (two's complement)
       uint64_t cy = 1;
       for (auto& w : np) { cy += (uint32_t)~w; w = (uint32_t)cy; cy >>= 32; }
-      R.o_tcE1 = ext(bytes_of(np, KB), 2 * KB);
-      R.o_tcE2 = ext(bytes_of(R.P2, KB), 3 * KB);
+      *e1 = ext(bytes_of(np, KB), KB, 2 * KB);
+      *e2 = ext(bytes_of(Nf, KB), KB, 3 * KB);
+    };
+    // (k_tc_exp starts from a table entry and needs at least one more schedule op: toy keys with
+    // one-window exponents stay on the CIOS kernels)
+    if ((sp == 32 || sp == 64) && V->pr[0].sched.ops.size() >= 2 && V->pr[1].sched.ops.size() >= 2) {
+      for (int i = 0; i < 2; i++) operands(V->pr[i].P2, sp, &V->pr[i].o_tcE1, &V->pr[i].o_tcE2);
+      V->tc = true;
     }
-    V->tc = true;
+    if (V->H == 32 || V->H == 64) {
+      for (int i = 0; i < 2; i++) operands(i == 0 ? V->p : V->q, V->H, &V->half[i].o_tcE1, &V->half[i].o_tcE2);
+      V->tc_half = true;
+    }
+    V->o_one = V->blob.put_raw(std::vector<uint32_t>{1u, 0u, 0u, 0u});
   }
   // CRT recombination constants
   H::MontCtx Cn(V->pub->n), Cp(V->p);
@@ -268,6 +280,25 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       *limb_products = (2 * per + 1) * csp + sp * sp;
       return FLB_OK;
     }
+    case 5: {  // key-holder encryption, tensor-core kernels (k_tc_exp) only: stage 1 at H, stage 2 at sp.
+      // Montgomery products on the tensor-core path; limb_products = the S^2 32x32-bit products of
+      // t = a b on the IMAD pipe (the reduction's u8 MACs are 32 S^2 per product: 2 MMAs of KB^2)
+      if (!V || !V->tc || !V->tc_half) return fail(FLB_EUNSUPPORTED, "no tensor-core key-holder path for this key");
+      const uint64_t h = V->H;
+      const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
+      const uint64_t s2 = (1 + sched_mults(V->sched_p) + 2) + (1 + sched_mults(V->sched_q) + 2);
+      *mont_muls = s1 + s2;
+      *limb_products = s1 * h * h + s2 * sp * sp;
+      return FLB_OK;
+    }
+    case 6: {  // decryption, tensor-core kernel (k_tc_exp) only: per prime 2 (entry) + table + schedule + 1
+      if (!V || !V->tc) return fail(FLB_EUNSUPPORTED, "no tensor-core decryption path for this key");
+      uint64_t mm = 0;
+      for (int i = 0; i < 2; i++) mm += 2 + sched_mults(V->pr[i].sched) + 1;
+      *mont_muls = mm;
+      *limb_products = mm * sp * sp;
+      return FLB_OK;
+    }
     case 2:
       *mont_muls = 2;
       *limb_products = 2 * cs;
@@ -362,12 +393,25 @@ int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t
   FLB_DISPATCH_ENC(K->frame, run_encrypt, K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 
+// tensor-core Montgomery paths (flb_tc.cuh): on when the key has the operands; FLB_TC=0 selects
+// the CIOS kernels (read per call, so tests can compare both)
+static bool tc_enabled() {
+  const char* e = getenv("FLB_TC");
+  return !(e && atoi(e) == 0);
+}
+static bool use_tc(const flb_priv* V) { return V->tc && tc_enabled(); }
+static bool use_tc_half(const flb_priv* V) { return V->tc_half && tc_enabled(); }
+
 int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count, void* stream) {
   if (!V || !c || !m) return fail(FLB_EINVAL, "null pointer");
   if (count == 0) return FLB_OK;
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
   if (rc) return rc;
+  if (use_tc(V)) {
+    if (V->pub->sp == 64) return run_decrypt_tc<64>(V, dev, c, m, count, (cudaStream_t)stream);
+    return run_decrypt_tc<32>(V, dev, c, m, count, (cudaStream_t)stream);
+  }
   FLB_DISPATCH_DEC(V->pub->frame, run_decrypt, V, dev, c, m, count, (cudaStream_t)stream);
 }
 
@@ -393,6 +437,14 @@ int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* 
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
   FLB_DISPATCH_ENC(K->frame, run_add_plain, K, dev, c1, c2, out, count, (cudaStream_t)stream);
+}
+
+int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, uint32_t words, int square,
+                         void* stream) {
+  if (!a || !b || !t || count > (uint32_t)flb::tc::kTileM) return fail(FLB_EINVAL, "null pointer or count > 128");
+  if (words == 64) return run_tc_debug_product<64>(a, b, t, count, square, (cudaStream_t)stream);
+  if (words == 32) return run_tc_debug_product<32>(a, b, t, count, square, (cudaStream_t)stream);
+  return fail(FLB_EINVAL, "words must be 32 or 64");
 }
 
 int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
@@ -651,20 +703,16 @@ static int crt2_dispatch(const flb_priv* V, const uint32_t* dev, const uint32_t*
   FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt2, V, dev, m, y, c, count, st);
 }
 
-// tensor-core Montgomery path for the key-holder stage 2 (flb_tc.cuh): on when the key has the
-// operands; FLB_TC=0 selects the CIOS kernel (read per call, so tests can compare both)
-static bool use_tc(const flb_priv* V) {
-  if (!V->tc) return false;
-  const char* e = getenv("FLB_TC");
-  return !(e && atoi(e) == 0);
-}
-
 static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
                           uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
   Scratch ys;
   int rc = ys.alloc((size_t)2 * count * V->H * 4, st);
   if (rc) return rc;
-  rc = crt_pre_dispatch(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
+  if (use_tc_half(V))
+    rc = V->H == 64 ? run_crt_pre_tc<64>(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st)
+                    : run_crt_pre_tc<32>(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
+  else
+    rc = crt_pre_dispatch(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
   if (rc) return rc;
   if (use_tc(V)) {
     if (V->pub->sp == 64) return run_encrypt_crt_tc<64>(V, dev, m, (const uint32_t*)ys.p, c, count, st);

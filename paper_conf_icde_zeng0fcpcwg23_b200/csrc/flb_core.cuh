@@ -126,7 +126,9 @@ struct flb_priv {
     // tensor-core Montgomery operands for P^2 (flb_tc.cuh): extended Toeplitz K-slices of N', N
     size_t o_tcE1 = 0, o_tcE2 = 0;
   } pr[2];
-  bool tc = false;  // tc operands present (sp in {32, 64})
+  bool tc = false;       // P^2 tensor-core operands present (sp in {32, 64})
+  bool tc_half = false;  // half-frame P tensor-core operands present (H in {32, 64})
+  size_t o_one = 0;      // the integer 1
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
   size_t o_q2invR = 0, o_enc_sched = 0;  // key-holder encryption: (q^2)^-1 R mod p^2, schedule of n
   // key-holder encryption v2 (r^n mod P^2 = (r^Q mod P)^P mod P^2): half-frame moduli and schedules
@@ -134,6 +136,7 @@ struct flb_priv {
   struct Half {
     uint32_t n0inv;
     size_t o_P, o_R2, o_R3;
+    size_t o_tcE1 = 0, o_tcE2 = 0;  // tensor-core operands of P in the H frame
   } half[2];
   H::Schedule sched_p, sched_q;           // exponents p and q
   size_t o_sched_p = 0, o_sched_q = 0;
@@ -493,52 +496,91 @@ int run_encrypt_crt2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, 
   return FLB_OK;
 }
 
-// key-holder stage 2 with the Montgomery reductions on the tensor cores (flb_tc.cuh): c_p and c_q
-// by k_tc_pow (one launch per prime), then k_crt_combine.
+// ----------------------------------------------------------------------------- tensor-core modexp
+// One k_tc_exp launch over the (up to two) problems of A: persistent grid of two 256-thread CTAs
+// per SM (flb_tc.cuh), window-table scratch sized for the largest table.
+template <int S>
+int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
+  using C = flb::tc::Cfg<S>;
+  int dev_id = 0, sms = 0;
+  FLB_CK(cudaGetDevice(&dev_id));
+  {
+    static std::mutex mu;
+    static std::map<int, bool> attr_done;  // function attributes are per device
+    std::lock_guard<std::mutex> lk(mu);
+    if (!attr_done[dev_id]) {
+      FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_exp<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+      FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_exp<S>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+      attr_done[dev_id] = true;
+    }
+  }
+  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id));
+  uint64_t tiles = 0;
+  int table = 1;
+  for (int i = 0; i < A.nprob; i++) {
+    auto& P = A.pb[i];
+    if (P.sched_len < 2) return fail(FLB_EUNSUPPORTED, "tensor-core path needs a multi-window exponent");
+    P.tiles = (P.count + flb::tc::kTileM - 1) / flb::tc::kTileM;
+    tiles += P.tiles;
+    table = std::max(table, P.table);
+  }
+  if (A.nprob < 2) A.pb[1].tiles = 0;
+  if (tiles == 0) return FLB_OK;
+  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), tiles);  // two CTAs per SM
+  Scratch s_tab;
+  int rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
+  if (rc) return rc;
+  A.scratch = (uint32_t*)s_tab.p;
+  A.tab_entries = table + 1;
+  flb::tc::k_tc_exp<S><<<grid, flb::tc::kThreads, C::SMEM, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+// debug: the tensor-core kernel's product phase alone (flb_debug_tc_product)
+template <int S>
+int run_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, int sq, cudaStream_t st) {
+  using C = flb::tc::Cfg<S>;
+  FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
+  flb::tc::k_tc_debug_product<S><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, sq);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+// key-holder stage 2 on the tensor cores: c_P = (1 + m n) y_P^P mod P^2 for both primes in one
+// k_tc_exp launch, then k_crt_combine
 template <int S>
 int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
                        size_t count, cudaStream_t st) {
-  using C = flb::tc::Cfg<S>;
-  static bool attr_done = false;
-  if (!attr_done) {
-    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_pow<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_pow<S>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-    attr_done = true;
-  }
-  int sms = 0, dev_id = 0;
-  FLB_CK(cudaGetDevice(&dev_id));
-  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id));
-  const uint64_t tiles = (count + flb::tc::kTileM - 1) / flb::tc::kTileM;
-  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), tiles);  // two CTAs per SM
-  const int table = std::max(V->sched_p.table, V->sched_q.table);
-  Scratch s_out, s_tab;
+  Scratch s_out;
   int rc = s_out.alloc((size_t)2 * count * S * 4, st);
   if (rc) return rc;
-  rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
-  if (rc) return rc;
   uint32_t* cpq = (uint32_t*)s_out.p;
+  flb::tc::ExpArgs A{};
+  A.nprob = 2;
+  A.one = dev + V->o_one;
   for (int i = 0; i < 2; i++) {
     const auto& R = V->pr[i];
     const H::Schedule& sc = i == 0 ? V->sched_p : V->sched_q;  // exponent P for P^2
-    flb::tc::PowArgs A;
-    A.P2 = dev + R.o_P2;
-    A.R2 = dev + R.o_R2;
-    A.nR = dev + R.o_nR;
-    A.E1 = dev + R.o_tcE1;
-    A.E2 = dev + R.o_tcE2;
-    A.sched = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
-    A.sched_len = (int)sc.ops.size();
-    if (A.sched_len < 2) return fail(FLB_EUNSUPPORTED, "tensor-core path needs a multi-window exponent");
-    A.table = sc.table;
-    A.y = y + (size_t)i * count * V->H;
-    A.H = V->H;
-    A.m = m;
-    A.out = cpq + (size_t)i * count * S;
-    A.count = count;
-    A.scratch = (uint32_t*)s_tab.p;
-    flb::tc::k_tc_pow<S><<<grid, flb::tc::kThreads, C::SMEM, st>>>(A);
-    FLB_LAUNCH_CHECK();
+    auto& P = A.pb[i];
+    P.N = dev + R.o_P2;
+    P.R2 = dev + R.o_R2;
+    P.R3 = dev + R.o_R3;
+    P.E1 = dev + R.o_tcE1;
+    P.E2 = dev + R.o_tcE2;
+    P.sched = dev + (i == 0 ? V->o_sched_p : V->o_sched_q);
+    P.sched_len = (int)sc.ops.size();
+    P.table = sc.table;
+    P.x = y + (size_t)i * count * V->H;
+    P.x_stride = V->H;
+    P.x_words = V->H;
+    P.m = m;
+    P.nR = dev + R.o_nR;
+    P.out = cpq + (size_t)i * count * S;
+    P.count = count;
   }
+  rc = launch_tc_exp<S>(A, st);
+  if (rc) return rc;
   constexpr int XC = 16, TC = S / 16;
   int cgrid;
   rc = grid_for<TC>(flb::k_crt_combine<XC, TC>, count, &cgrid);
@@ -552,6 +594,112 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
   B.c = c;
   B.count = count;
   flb::k_crt_combine<XC, TC><<<cgrid, kBlock, 0, st>>>(B);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+// key-holder stage 1 on the tensor cores: y_P = r^Q mod P in the H-word frame (both primes, one
+// launch); r drawn by k_philox_fill unless the caller passes it
+template <int HS>
+int run_crt_pre_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0,
+                   uint32_t* y, size_t count, cudaStream_t st) {
+  const uint32_t sp = V->pub->sp;
+  Scratch s_r;
+  if (!r) {
+    int rc = s_r.alloc((size_t)count * sp * 4, st);
+    if (rc) return rc;
+    int g;
+    switch (sp) {
+#define FLB_FILL(SPW)                                                                          \
+  case SPW:                                                                                    \
+    rc = grid_for<4>(flb::k_philox_fill<SPW / 4, 4>, count, &g); /* groups of 4 lanes (T a power of 2) */ \
+    if (rc) return rc;                                                                         \
+    flb::k_philox_fill<SPW / 4, 4><<<g, kBlock, 0, st>>>((uint32_t*)s_r.p, count, V->pub->nbits, seed, ctr0); \
+    break;
+      FLB_FILL(64)
+      FLB_FILL(96)
+      FLB_FILL(128)
+#undef FLB_FILL
+      default:
+        return fail(FLB_EUNSUPPORTED, "tensor-core stage 1: unsupported plaintext frame");
+    }
+    FLB_LAUNCH_CHECK();
+    r = (const uint32_t*)s_r.p;
+  }
+  flb::tc::ExpArgs A{};
+  A.nprob = 2;
+  A.one = dev + V->o_one;
+  for (int i = 0; i < 2; i++) {
+    const H::Schedule& sc = i == 0 ? V->sched_q : V->sched_p;  // exponent: the other prime
+    auto& P = A.pb[i];
+    P.N = dev + V->half[i].o_P;
+    P.R2 = dev + V->half[i].o_R2;
+    P.R3 = dev + V->half[i].o_R3;
+    P.E1 = dev + V->half[i].o_tcE1;
+    P.E2 = dev + V->half[i].o_tcE2;
+    P.sched = dev + (i == 0 ? V->o_sched_q : V->o_sched_p);
+    P.sched_len = (int)sc.ops.size();
+    P.table = sc.table;
+    P.x = r;
+    P.x_stride = sp;
+    P.x_words = sp;
+    P.m = nullptr;
+    P.out = y + (size_t)i * count * HS;
+    P.count = count;
+  }
+  return launch_tc_exp<HS>(A, st);
+}
+
+// decryption with both exponentiations c^(P-1) mod P^2 on the tensor cores (one launch), then the
+// CRT tail k_dec_finish on the CUDA cores
+template <int S>
+int run_decrypt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* c, uint32_t* m, size_t count,
+                   cudaStream_t st) {
+  Scratch s_x;
+  int rc = s_x.alloc((size_t)2 * count * S * 4, st);
+  if (rc) return rc;
+  uint32_t* xp = (uint32_t*)s_x.p;
+  flb::tc::ExpArgs A{};
+  A.nprob = 2;
+  A.one = dev + V->o_one;
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    auto& P = A.pb[i];
+    P.N = dev + R.o_P2;
+    P.R2 = dev + R.o_R2;
+    P.R3 = dev + R.o_R3;
+    P.E1 = dev + R.o_tcE1;
+    P.E2 = dev + R.o_tcE2;
+    P.sched = dev + R.o_sched;  // exponent P - 1
+    P.sched_len = (int)R.sched.ops.size();
+    P.table = R.sched.table;
+    P.x = c;
+    P.x_stride = 2 * S;
+    P.x_words = 2 * S;
+    P.m = nullptr;
+    P.out = xp + (size_t)i * count * S;
+    P.count = count;
+  }
+  rc = launch_tc_exp<S>(A, st);
+  if (rc) return rc;
+  constexpr int XF = 16, TF = S / 16;
+  int grid;
+  rc = grid_for<TF>(flb::k_dec_finish<XF, TF>, count, &grid);
+  if (rc) return rc;
+  flb::DecArgs D{};
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    D.pr[i].P = {dev + R.o_P, R.P_n0inv};
+    D.pr[i].Pinv = dev + R.o_Pinv;
+    D.pr[i].hR = dev + R.o_hR;
+  }
+  D.n = {dev + V->o_n, V->n_n0inv};
+  D.qR_n = dev + V->o_qR_n;
+  D.qinvR_p = dev + V->o_qinvR_p;
+  D.xp = xp;
+  D.m = m;
+  D.count = count;
+  flb::k_dec_finish<XF, TF><<<grid, kBlock, 0, st>>>(D);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }
@@ -714,7 +862,13 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
                                                   const uint32_t*, uint32_t*, size_t, cudaStream_t);
 #define FLB_TC_DECLS(EXT, S)                                                                                      \
   EXT template int flb_rt::run_encrypt_crt_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*,              \
-                                                 const uint32_t*, uint32_t*, size_t, cudaStream_t);
+                                                 const uint32_t*, uint32_t*, size_t, cudaStream_t);              \
+  EXT template int flb_rt::run_crt_pre_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*, uint64_t,        \
+                                             uint64_t, uint32_t*, size_t, cudaStream_t);                        \
+  EXT template int flb_rt::run_decrypt_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*, uint32_t*,       \
+                                             size_t, cudaStream_t);                                              \
+  EXT template int flb_rt::run_tc_debug_product<S>(const uint32_t*, const uint32_t*, uint32_t*, uint32_t, int,   \
+                                                   cudaStream_t);
 
 #ifndef FLB_INST_TU
 #define FLB_EXTERN_ENC(X, T) FLB_ENC_DECLS(extern, X, T)

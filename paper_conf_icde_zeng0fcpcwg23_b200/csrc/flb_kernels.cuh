@@ -226,6 +226,7 @@ struct DecArgs {
   uint32_t* m;            // [count][sp]
   uint64_t count;
   uint32_t* scratch;      // max table * G * sp
+  const uint32_t* xp;     // k_dec_finish: [2][count][sp], c^(P-1) mod P^2 (canonical)
 };
 
 // m = D(c) (Eq. 4) by CRT (reading c10):
@@ -1202,4 +1203,63 @@ __global__ void __launch_bounds__(32, FLB_MINB_MUL) k_crt_combine(const CombineA
     }
   }
 }
+// The CRT tail of k_decrypt after the two exponentiations (done on the tensor cores, flb_tc.cuh
+// k_tc_exp): from x_P = c^(P-1) mod P^2, m_P = L_P(x_P) h_P mod P and
+// m = m_q + q ((m_p - m_q) q^-1 mod p) (Eq. 4 by CRT, reading c10).
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_dec_finish(const DecArgs A) {
+  constexpr int S = X * T;  // sp
+  const Grid<T> g;
+  for (uint64_t base = g.wg0; base < A.count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    const bool valid = e < A.count;
+    uint32_t mres[2][X];
+#pragma unroll 1
+    for (int P = 0; P < 2; P++) {
+      const PrimeArgs& pa = A.pr[P];
+      uint32_t n[X], lo[X], hi[X], b[X];
+      load_elem<X, T>(lo, A.xp + ((uint64_t)P * A.count + e) * S, S, valid);
+      grp_sub_one<X, T>(lo);                              // x - 1 = L * P
+      load_const<X, T>(b, pa.Pinv);
+      mul_lo<X, T>(hi, lo, b);                            // L = (x - 1) / P (exact division)
+      load_mod<X, T>(n, pa.P);
+      load_const<X, T>(b, pa.hR);
+      mont_mul<X, T>(lo, hi, b, n, pa.P.n0inv);           // m_P = L h_P mod P
+#pragma unroll
+      for (int j = 0; j < X; j++) {
+        if (P == 0) mres[0][j] = lo[j];
+        else mres[1][j] = lo[j];
+      }
+    }
+    uint32_t n[X], d[X], t[X];
+    load_mod<X, T>(n, A.pr[0].P);
+    const uint32_t br = grp_sub<X, T>(d, mres[0], mres[1]);   // m_p - m_q (m_q < q < p)
+#pragma unroll
+    for (int j = 0; j < X; j++) t[j] = br ? n[j] : 0u;
+    grp_add<X, T>(d, d, t);                                    // mod p
+    load_const<X, T>(t, A.qinvR_p);
+    mont_mul<X, T>(d, d, t, n, A.pr[0].P.n0inv);               // u = (m_p - m_q) q^-1 mod p
+    load_mod<X, T>(n, A.n);
+    load_const<X, T>(t, A.qR_n);
+    mont_mul<X, T>(d, d, t, n, A.n.n0inv);                     // q u (< n, exact)
+    grp_add<X, T>(d, d, mres[1]);                              // m = m_q + q u
+    if (valid) store_limbs<X>(A.m + e * S + g.k * X, d);
+  }
+}
+
+// r for elements [0, count) as k_encrypt draws it (philox_r, reading c4) into [count][pt_words],
+// X T = pt_words: the input of the tensor-core first stage of the key-holder encryption.
+template <int X, int T>
+__global__ void __launch_bounds__(32, FLB_MINB_MUL) k_philox_fill(uint32_t* __restrict__ r, uint64_t count,
+                                                                  uint32_t nbits, uint64_t seed, uint64_t ctr0) {
+  constexpr int S = X * T;
+  const Grid<T> g;
+  for (uint64_t base = g.wg0; base < count; base += g.G) {
+    const uint64_t e = base + (g.gid - g.wg0);
+    uint32_t v[X];
+    philox_r<X, T>(v, seed, ctr0 + e, S, nbits);
+    if (e < count) store_limbs<X>(r + e * S + g.k * X, v);
+  }
+}
 }  // namespace flb
+

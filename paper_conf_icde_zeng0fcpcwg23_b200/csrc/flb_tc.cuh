@@ -190,25 +190,163 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
   }
 }
 
-// Montgomery product over the tile: for every element, a b R^-1 mod N (canonical) into its work
-// row.  sq: b = a.  `phase` tracks the mbarrier parity (two completions per call).  CTA-collective.
-template <int S>
-__device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, const Smem& sm,
-                                        const uint32_t* __restrict__ Nmod, uint32_t& phase) {
-  using C = Cfg<S>;
-  constexpr int X = C::X, KCH = C::KCH, KB = C::KB, QW = C::QW, QC = C::QC;
-  const int tid = threadIdx.x, k = tid % kT, warp = tid >> 5;
-  uint8_t* sA = sm.base + C::OFF_A;
-  uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
-#if FLB_TC_PROF
-  long long t_ = clock64();
+#ifndef FLB_TC_SQR
+#define FLB_TC_SQR 1  // block squaring in the product phase (0: squarings use the general product)
 #endif
+
+// ----------------------------------------------------------------------------- squaring product
+// t = a^2 for the product phase when a = b (87 % of the multiplications of a modexp).  Lane k of the
+// element's group holds the limb block a_k = a[kX, kX+X) (X = S/4).  a^2 is the sum of block
+// products a_i a_j 2^(32 X (i+j)) over i <= j, the off-diagonal ones doubled; each lane computes
+// the same shapes (so the warp never diverges in the multiply code): its diagonal block a_k a_k
+// (X x X), one full off-diagonal block a_k a_(k+1 mod 4) (X x X), and half of a_(k&1) a_(k&1)+2
+// (X x X/2, row half k>>1): X^2 + X^2 + X^2/2 = 2.5 X^2 = 640 limb products at S = 64 instead of the
+// general product's S X = 1024.  Row words of another lane's block arrive by shuffle.  The pieces
+// are accumulated in place in t's destination rows (t_lo: the element's sA row, the MMA operand;
+// t_hi: its work row) in phases with disjoint word ranges, their carry-outs folded in by one final
+// group pass with a ballot carry-lookahead.
+template <int X, int R>
+__device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t (&M)[X], const uint32_t (&a)[X],
+                                         int src, bool own_upper) {
+  // out = M x (R row words of lane src's block): words [0, R) of it by shuffle (every lane serves its
+  // own a[j]), or, with own_upper (src is this lane), this lane's words [R, 2R) directly
+  uint32_t E[X + 1], O[X + 1], pend = 0;
+#pragma unroll
+  for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
+#pragma unroll
+  for (int j = 0; j < R; j++) {
+    uint32_t bj = __shfl_sync(FULL, a[j], src, kT);
+    if (R < X && own_upper) bj = a[(j + R) % X];
+    out[j] = local_row<X>(E, O, pend, M, bj);
+  }
+  asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(out[R]) : "r"(E[0]), "r"(pend));
+#pragma unroll
+  for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(out[R + t]) : "r"(E[t]), "r"(O[t - 1]));
+}
+
+// address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work row
+template <int S>
+__device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, int w) {
+  using C = Cfg<S>;
+  return w < S ? reinterpret_cast<uint4*>(sA + cm_off(elem, 4u * w, C::KCH))
+               : reinterpret_cast<uint4*>(sW + elem * C::WROW + (w - S));
+}
+
+// t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2)
+template <int S, int NW>
+__device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int elem, int w0, const uint32_t (&v)[NW]) {
+  uint64_t cy = 0;
+  uint32_t prev = 0;
+#pragma unroll
+  for (int c = 0; c < NW / 4; c++) {
+    uint4* p = t_chunk<S>(sA, sW, elem, w0 + 4 * c);
+    const uint4 m = *p;
+    uint32_t d[4], r[4];
+    const uint32_t mm[4] = {m.x, m.y, m.z, m.w};
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t x = v[4 * c + u];
+      d[u] = (x << 1) | (prev >> 31);
+      prev = x;
+      const uint64_t s = (uint64_t)mm[u] + d[u] + cy;
+      r[u] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    *p = make_uint4(r[0], r[1], r[2], r[3]);
+  }
+  return (uint32_t)cy + (prev >> 31);
+}
+
+template <int S>
+__device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
+                                                  uint32_t* sW) {
+  constexpr int X = Cfg<S>::X, H = X / 2;
+  const int k = threadIdx.x % kT;
+  uint32_t cF = 0, cH = 0;
+  {
+    // diagonal block: t[2Xk, 2Xk + 2X) = a_k^2 (the four tile t exactly)
+    uint32_t v[2 * X];
+    blk_prod<X, X>(v, a, a, k, false);
+    __syncwarp();  // every lane of the group has read its a (it may come from the work row)
+#pragma unroll
+    for (int c = 0; c < X / 2; c++)
+      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  }
+  {
+    // full off-diagonal block a_k a_l, l = k + 1 mod 4, doubled, at words X (k + l) (lane 3: X 3)
+    uint32_t v[2 * X];
+    const int l = (k + 1) & (kT - 1);
+    blk_prod<X, X>(v, a, a, l, false);
+    const int w0 = X * (k < kT - 1 ? 2 * k + 1 : kT - 1);
+    __syncwarp();
+    if (k < kT - 1) cF = t_add_dbl<S, 2 * X>(sA, sW, elem, w0, v);  // [X, 3X), [3X, 5X), [5X, 7X)
+    __syncwarp();
+    if (k == kT - 1) cF = t_add_dbl<S, 2 * X>(sA, sW, elem, w0, v);  // [3X, 5X)
+  }
+  {
+    // half block: a_(k&1) x a_((k&1)+2)[H (k>>1), + H), doubled, at words 2X (k&1) + 2X + H (k>>1)
+    uint32_t M[X], v[X + H];
+    const int i = k & 1, hh = k >> 1;
+#pragma unroll
+    for (int j = 0; j < X; j++) M[j] = __shfl_sync(FULL, a[j], i, kT);
+    // rows [0, H) of a_(i+2) come from lane i + 2 (read by lane i); lane i + 2 itself (hh = 1) takes
+    // its own rows [H, X)
+    blk_prod<X, H>(v, M, a, i + 2, hh == 1);
+    const int w0 = 2 * X * i + 2 * X + H * hh;
+    __syncwarp();
+    if (hh == 0) cH = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);  // [2X, 3.5X), [4X, 5.5X)
+    __syncwarp();
+    if (hh == 1) cH = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);  // [2.5X, 4X), [4.5X, 6X)
+    __syncwarp();
+  }
+  // fold the carries into lane k's quarter [2Xk, 2Xk + 2X): at relative offsets 0, X, 1.5X
+  //   q1: X <- cF(0), 1.5X <- cH(0);  q2: 0 <- cH(2), X <- cF(1) + cF(3), 1.5X <- cH(1);
+  //   q3: 0 <- cH(3), X <- cF(2)
+  const uint32_t f0 = __shfl_sync(FULL, cF, 0, kT), f1 = __shfl_sync(FULL, cF, 1, kT);
+  const uint32_t f2 = __shfl_sync(FULL, cF, 2, kT), f3 = __shfl_sync(FULL, cF, 3, kT);
+  const uint32_t h0 = __shfl_sync(FULL, cH, 0, kT), h1 = __shfl_sync(FULL, cH, 1, kT);
+  const uint32_t at0 = k >= 2 ? cH : 0u;
+  const uint32_t atX = k == 1 ? f0 : k == 2 ? f1 + f3 : k == 3 ? f2 : 0u;
+  const uint32_t atH = k == 1 ? h0 : k == 2 ? h1 : 0u;
+  uint32_t q[2 * X];
+#pragma unroll
+  for (int c = 0; c < X / 2; c++) {
+    const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c);
+    q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
+  }
+  uint64_t cy = 0;
+#pragma unroll
+  for (int j = 0; j < 2 * X; j++) {
+    const uint32_t add = j == 0 ? at0 : j == X ? atX : j == X + H ? atH : 0u;
+    const uint64_t s = (uint64_t)q[j] + add + cy;
+    q[j] = (uint32_t)s;
+    cy = s >> 32;
+  }
+  const uint32_t c = group_carry<kT>(cy != 0, all_ones<2 * X>(q), 0);
+  add_word_propagate<2 * X>(q, c & 1u);
+#pragma unroll
+  for (int cc = 0; cc < X / 2; cc++)
+    *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
+}
+
+// The product phase of tc_mont: t = a b (2S words) for the 128 elements of the tile, t_lo into the
+// elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of kT lanes per element,
+// two halves of 64 elements.  CTA-collective (no trailing barrier).
+template <int S>
+__device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq, uint8_t* sA, uint32_t* sW) {
+  using C = Cfg<S>;
+  constexpr int X = C::X, KCH = C::KCH;
+  const int tid = threadIdx.x, k = tid % kT;
   // ---- P: t = a b, two halves of 64 elements
 #pragma unroll 1
   for (int h = 0; h < 2; h++) {
     const int elem = h * kHalf + tid / kT;
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
+    if (FLB_TC_SQR && S >= 64 && sq) {  // measured: a gain at S = 64, a loss at S = 32
+      tc_square_product<S>(a, elem, sA, sW);
+      continue;
+    }
     if (sq) {
 #pragma unroll
       for (int j = 0; j < X; j++) b[j] = a[j];
@@ -251,6 +389,22 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
           make_uint4(hi[4 * v], hi[4 * v + 1], hi[4 * v + 2], hi[4 * v + 3]);
     }
   }
+}
+
+// Montgomery product over the tile: for every element, a b R^-1 mod N (canonical) into its work
+// row.  sq: b = a.  `phase` tracks the mbarrier parity (two completions per call).  CTA-collective.
+template <int S>
+__device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, const Smem& sm,
+                                        const uint32_t* __restrict__ Nmod, uint32_t& phase) {
+  using C = Cfg<S>;
+  constexpr int X = C::X, KCH = C::KCH, KB = C::KB, QW = C::QW, QC = C::QC;
+  const int tid = threadIdx.x, k = tid % kT, warp = tid >> 5;
+  uint8_t* sA = sm.base + C::OFF_A;
+  uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
+#if FLB_TC_PROF
+  long long t_ = clock64();
+#endif
+  tc_product<S>(sa, sb, sq, sA, sW);
   fence_async_smem();
   tc_before_sync();
   __syncthreads();
@@ -482,43 +636,83 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
   __syncthreads();
 }
 
-// ----------------------------------------------------------------------------- key-holder stage 2
-// c_P = (1 + m n) y^P mod P^2 for one prime P per launch (Eq. 3 with g = n + 1, by the
-// two-stage CRT of k_encrypt_crt2: y = r^Q mod P from k_crt_pre), every Montgomery product by
-// tc_mont.  Persistent CTAs over 128-element tiles; the odd-power window table of each element
-// lives in global scratch [entry][elem][S] per CTA (entry `table` holds x^2, then the saved power).
-struct PowArgs {
-  const uint32_t* P2;      // modulus P^2 (S words)
-  const uint32_t* R2;      // R^2 mod P^2
-  const uint32_t* nR;      // n R mod P^2
+// work row <- (row + s) mod N for every element (row, s < N)
+template <int S>
+__device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const uint32_t* __restrict__ Nmod) {
+  using C = Cfg<S>;
+  constexpr int X = C::X;
+  uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
+  const int k = threadIdx.x % kT;
+#pragma unroll 1
+  for (int h = 0; h < 2; h++) {
+    const int elem = h * kHalf + threadIdx.x / kT;
+    uint32_t r[X], a[X], nn[X];
+    src_load<S>(r, src_row(), elem, sW);
+    src_load<S>(a, s, elem, sW);
+    load_const<X, kT>(nn, Nmod);
+    const uint32_t cy = grp_add<X, kT>(r, r, a);
+    grp_cond_sub<X, kT>(r, nn, cy);
+    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + k * X);
+#pragma unroll
+    for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
+  }
+  __syncthreads();
+}
+
+// ----------------------------------------------------------------------------- batched modexp
+// One modular exponentiation per element with an exponent shared by the batch (the
+// windowed modexp of Alg. 2's Montgomery product), every Montgomery product by tc_mont.  A launch
+// serves up to two problems (the two CRT primes); its tiles are numbered problem 0 first, and a
+// persistent CTA reloads the Toeplitz operands when it crosses into the other problem.
+//   input  x: x_words <= S words per element (x R = mont(x, R^2)), or 2S words split as lo + hi R
+//         (x R = mont(lo, R^2) + mont(hi, R^3)), i.e. a 2S-word integer entering the S-word frame
+//   output m == null: x^E mod N (canonical);  m != null: (1 + m n) x^E mod N (Eq. 3,
+//         g = n + 1, for the key-holder encryption with x = r^Q mod P and E = P)
+// The odd-power window table of each element lives in global scratch [entry][elem][S] per CTA
+// (entry `table` holds x^2, then the saved power).
+struct ExpProblem {
+  const uint32_t* N;       // modulus (S words)
+  const uint32_t* R2;      // R^2 mod N
+  const uint32_t* R3;      // R^3 mod N (two-half input only)
   const uint32_t* E1;      // extended Toeplitz(N') operand, 2KB x 32 bytes (core matrices)
   const uint32_t* E2;      // extended Toeplitz(N) operand, 3KB x 32 bytes
-  const uint32_t* sched;   // schedule of the exponent P (at least one op after the first window)
+  const uint32_t* sched;   // exponent schedule (at least one op after the first window)
   int sched_len, table;
-  const uint32_t* y;       // [count][H]
-  uint32_t H;
-  const uint32_t* m;       // [count][S]
+  const uint32_t* x;       // [count][x_stride]
+  uint32_t x_stride, x_words;
+  const uint32_t* m;       // [count][S] or null
+  const uint32_t* nR;      // n R mod N (with m)
   uint32_t* out;           // [count][S]
-  uint64_t count;
-  uint32_t* scratch;       // gridDim * kTileM * (table + 1) * S words
+  uint64_t count, tiles;
+};
+struct ExpArgs {
+  ExpProblem pb[2];
+  int nprob;
+  const uint32_t* one;     // the integer 1 (at least one word)
+  uint32_t* scratch;       // gridDim * kTileM * tab_entries * S words
+  int tab_entries;         // max table over the problems + 1 (the per-CTA scratch stride)
 };
 
 template <int S>
-__global__ void __launch_bounds__(kThreads, 2) k_tc_pow(const PowArgs A) {
+__device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem& P) {
   using C = Cfg<S>;
   constexpr int KB = C::KB;
+  const uint4* s1 = reinterpret_cast<const uint4*>(P.E1);
+  const uint4* s2 = reinterpret_cast<const uint4*>(P.E2);
+  uint4* d1 = reinterpret_cast<uint4*>(smem + C::OFF_E1);
+  uint4* d2 = reinterpret_cast<uint4*>(smem + C::OFF_E2);
+  for (int i = threadIdx.x; i < 2 * KB * 32 / 16; i += kThreads) d1[i] = __ldg(s1 + i);
+  for (int i = threadIdx.x; i < 3 * KB * 32 / 16; i += kThreads) d2[i] = __ldg(s2 + i);
+  fence_async_smem();
+}
+
+template <int S>
+__global__ void __launch_bounds__(kThreads, 2) k_tc_exp(const ExpArgs A) {
+  using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t tmem_sh;
   const int tid = threadIdx.x, warp = tid >> 5;
-  {
-    const uint4* s1 = reinterpret_cast<const uint4*>(A.E1);
-    const uint4* s2 = reinterpret_cast<const uint4*>(A.E2);
-    uint4* d1 = reinterpret_cast<uint4*>(smem + C::OFF_E1);
-    uint4* d2 = reinterpret_cast<uint4*>(smem + C::OFF_E2);
-    for (int i = tid; i < 2 * KB * 32 / 16; i += kThreads) d1[i] = __ldg(s1 + i);
-    for (int i = tid; i < 3 * KB * 32 / 16; i += kThreads) d2[i] = __ldg(s2 + i);
-  }
   if (tid == 0) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&mbar)));
     asm volatile("fence.mbarrier_init.release.cluster;");
@@ -528,52 +722,76 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_pow(const PowArgs A) {
                  "n"(C::TMEM_COLS));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
-  fence_async_smem();
   tc_before_sync();
   __syncthreads();
   tc_after_sync();
   const Smem sm{smem, tmem_sh, &mbar};
   uint32_t phase = 0;
-  const int TB = A.table;
-  uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * (TB + 1) * S;
-  auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
-  auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
+  const uint64_t tiles_all = A.pb[0].tiles + (A.nprob > 1 ? A.pb[1].tiles : 0);
+  int loaded = -1;
   const Src row = src_row();
-  for (uint64_t tile = blockIdx.x; tile * kTileM < A.count; tile += gridDim.x) {
+  for (uint64_t gt = blockIdx.x; gt < tiles_all; gt += gridDim.x) {
+    const int pi = gt < A.pb[0].tiles ? 0 : 1;
+    const ExpProblem& P = A.pb[pi];
+    const uint64_t tile = pi == 0 ? gt : gt - A.pb[0].tiles;
+    if (pi != loaded) {
+      __syncthreads();  // the previous problem's MMAs completed (waited on) before the overwrite
+      tc_load_operands<S>(smem, P);
+      tc_before_sync();
+      __syncthreads();
+      loaded = pi;
+    }
+    const int TB = P.table;
+    uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * A.tab_entries * S;
+    auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
+    auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
     const uint64_t e0 = tile * kTileM;
-    const uint32_t nvalid = (uint32_t)((A.count - e0) < (uint64_t)kTileM ? (A.count - e0) : (uint64_t)kTileM);
-    tc_mont<S>(src_arr(A.y + e0 * A.H, A.H, A.H, nvalid), src_arr(A.R2, 0, S, kTileM), false, sm, A.P2, phase);
-    tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x = y R mod P^2
+    const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
+    const uint32_t* xb = P.x + e0 * P.x_stride;
+    if (P.x_words <= (uint32_t)S) {
+      tc_mont<S>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    } else {
+      tc_mont<S>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+      tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
+      tc_mont<S>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
+                 phase);                                      // hi R^2
+      tc_row_add<S>(sm, slot(0), P.N);
+    }
+    tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
     if (TB > 1) {
-      tc_mont<S>(row, row, true, sm, A.P2, phase);            // x^2
+      tc_mont<S>(row, row, true, sm, P.N, phase);             // x^2
       tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
 #pragma unroll 1
       for (int t = 1; t < TB; t++) {
-        tc_mont<S>(slot(t - 1), slot(TB), false, sm, A.P2, phase);
+        tc_mont<S>(slot(t - 1), slot(TB), false, sm, P.N, phase);
         tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
       }
     }
-    const uint32_t op0 = __ldg(A.sched);
+    const uint32_t op0 = __ldg(P.sched);
     Src cur = slot((int)(op0 >> 16) - 1);
 #pragma unroll 1
-    for (int o = 1; o < A.sched_len; o++) {
-      const uint32_t op = __ldg(A.sched + o);
+    for (int o = 1; o < P.sched_len; o++) {
+      const uint32_t op = __ldg(P.sched + o);
       const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
 #pragma unroll 1
       for (int t = 0; t < sq; t++) {
-        tc_mont<S>(cur, cur, true, sm, A.P2, phase);
+        tc_mont<S>(cur, cur, true, sm, P.N, phase);
         cur = row;
       }
       if (idx >= 0) {
-        tc_mont<S>(cur, slot(idx), false, sm, A.P2, phase);
+        tc_mont<S>(cur, slot(idx), false, sm, P.N, phase);
         cur = row;
       }
     }
-    tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);             // y^P R
-    tc_mont<S>(src_arr(A.m + e0 * S, S, S, nvalid), src_arr(A.nR, 0, S, kTileM), false, sm, A.P2, phase);  // m n
-    tc_row_add_one<S>(sm, A.P2);                              // 1 + m n mod P^2
-    tc_mont<S>(slot(TB), row, false, sm, A.P2, phase);        // c_P
-    tc_row_store<S>(sm, A.out + e0 * S, S, nvalid);
+    if (P.m) {
+      tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
+      tc_mont<S>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
+      tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
+      tc_mont<S>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
+    } else {
+      tc_mont<S>(row, src_arr(A.one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
+    }
+    tc_row_store<S>(sm, P.out + e0 * S, S, nvalid);
     __syncthreads();  // the work rows are rewritten by the next tile's first product
   }
   tc_before_sync();
@@ -581,6 +799,22 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_pow(const PowArgs A) {
   if (warp == 0) {
     tc_after_sync();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem_sh), "n"(C::TMEM_COLS));
+  }
+}
+
+// debug: the product phase alone (t = a b, or a^2 when sq) for up to 128 elements -> t [count][2S]
+template <int S>
+__global__ void __launch_bounds__(kThreads, 1) k_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t,
+                                                                  uint32_t count, int sq) {
+  using C = Cfg<S>;
+  extern __shared__ __align__(1024) uint8_t smem[];
+  uint8_t* sA = smem + C::OFF_A;
+  uint32_t* sW = reinterpret_cast<uint32_t*>(smem + C::OFF_W);
+  tc_product<S>(src_arr(a, S, S, count), src_arr(b, S, S, count), sq != 0, sA, sW);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < count * 2 * S; i += kThreads) {
+    const uint32_t e = i / (2 * S), w = i % (2 * S);
+    t[i] = w < (uint32_t)S ? *reinterpret_cast<const uint32_t*>(sA + cm_off(e, 4u * w, C::KCH)) : sW[e * C::WROW + w - S];
   }
 }
 

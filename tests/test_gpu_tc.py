@@ -79,3 +79,114 @@ def test_tc_large_batch_matches_cios(k2048):
     cios, tc = _both(priv, m, seed=0xABCDEF, ctr0=1 << 33)
     bad = (cios != tc).any(dim=1).nonzero().flatten().tolist()
     assert not bad, bad[:5]
+
+
+def _both_dec(priv, c):
+    old = os.environ.get("FLB_TC")
+    try:
+        os.environ["FLB_TC"] = "0"
+        cios = flb.decrypt(priv, c)
+        os.environ["FLB_TC"] = "1"
+        tc = flb.decrypt(priv, c)
+    finally:
+        if old is None:
+            os.environ.pop("FLB_TC", None)
+        else:
+            os.environ["FLB_TC"] = old
+    torch.cuda.synchronize()
+    return cios, tc
+
+
+@pytest.mark.parametrize("bits", ["1024", "2048"])
+@pytest.mark.parametrize("count", [1, 129, 300])
+def test_tc_decrypt_matches_cios_and_oracle(bits, count):
+    """Decryption with c^(P-1) mod P^2 on the tensor cores (k_tc_exp + k_dec_finish): the same
+    plaintexts as the CIOS k_decrypt and as the oracle's literal Eq. 4."""
+    p, q = KEYS[bits]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    m_int = synthetic.uniform_below(n, count, 900 + count)
+    m_int[0] = 0
+    if count > 1:
+        m_int[-1] = n - 1
+    seed = 0x7D000000 + count
+    c = flb.encrypt(pub, to_dev(m_int, pub.pt_words), seed=seed)
+    cios, tc = _both_dec(priv, c)
+    assert torch.equal(cios, tc)
+    got = from_dev(tc)
+    assert got == m_int
+    cc = from_dev(c)
+    for i in sorted({0, count // 2, count - 1}):
+        assert paillier.decrypt(p, q, cc[i]) == m_int[i], i
+
+
+def test_tc_decrypt_arbitrary_ciphertexts_match_cios():
+    """Any 2S-word c < n^2 (not only encryptions): both CRT exponentiation paths agree bit for bit."""
+    p, q = KEYS["2048"]
+    pub, priv = flb.key_from_primes(p, q)
+    n2 = (p * q) ** 2
+    cs = synthetic.uniform_below(n2, 1000, 4242)
+    cs[:3] = [1, n2 - 1, p * p]
+    c = to_dev(cs, pub.ct_words)
+    cios, tc = _both_dec(priv, c)
+    bad = (cios != tc).any(dim=1).nonzero().flatten().tolist()
+    assert not bad, bad[:5]
+
+
+@pytest.mark.parametrize("bits", ["3072", "4096"])
+def test_tc_stage1_large_keys_match_cios_and_oracle(bits):
+    """Key-holder stage 1 (r^Q mod P in the 64-word half frame) on the tensor cores at 3072/4096
+    bits, stage 2 on CIOS: same ciphertexts as FLB_TC=0 and as the oracle's Eq. 3."""
+    p, q = KEYS[bits]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    count = 130
+    m_int = synthetic.uniform_below(n, count, 77)
+    m = to_dev(m_int, pub.pt_words)
+    cios, tc = _both(priv, m, seed=0x51, ctr0=5)
+    assert torch.equal(cios, tc)
+    got = from_dev(tc)
+    for i in (0, 64, 129):
+        assert got[i] == paillier.encrypt(n, m_int[i], philox.draw_r(n, 0x51, 5 + i, pub.pt_words)), i
+
+
+def test_tc_multi_tile_per_cta_both_problems():
+    """Batches larger than one round of the persistent grid (every CTA runs several tiles and
+    crosses from the p problem into the q problem, whose window tables differ in size at 1024
+    bits): decryption and key-holder encryption equal the CIOS kernels bit for bit."""
+    p, q = KEYS["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    count = 40000
+    m_int = synthetic.uniform_below(n, count, 31337)
+    m = to_dev(m_int, pub.pt_words)
+    c = flb.encrypt(pub, m, seed=0x99)
+    cios, tc = _both_dec(priv, c)
+    assert torch.equal(cios, tc)
+    assert torch.equal(tc, m)
+    p2, q2 = KEYS["2048"]
+    pub2, priv2 = flb.key_from_primes(p2, q2)
+    m2 = to_dev(synthetic.uniform_below(p2 * q2, count, 4711), pub2.pt_words)
+    cios_e, tc_e = _both(priv2, m2, seed=0x98, ctr0=3)
+    assert torch.equal(cios_e, tc_e)
+    cios_d, tc_d = _both_dec(priv2, tc_e)
+    assert torch.equal(cios_d, tc_d)
+    assert torch.equal(tc_d, m2)
+
+
+@pytest.mark.parametrize("words", [32, 64])
+@pytest.mark.parametrize("square", [False, True])
+def test_tc_product_phase_exact(words, square):
+    """The tensor-core kernel's CUDA-core product phase (general row scan, or the block squaring
+    of a^2) gives the exact 2w-limb integer product on random and extreme operands."""
+    count = 128
+    rnd = synthetic.uniform_below(1 << (32 * words), count, 5150 + words + square)
+    top = (1 << (32 * words)) - 1
+    rnd[:6] = [0, 1, top, top - 1, 1 << (32 * words - 1), (1 << (16 * words)) - 1]
+    other = synthetic.uniform_below(1 << (32 * words), count, 6150 + words)
+    a = to_dev(rnd, words)
+    b = to_dev(other, words)
+    t = from_dev(flb.debug_tc_product(a, b, square=square))
+    for i in range(count):
+        want = rnd[i] * (rnd[i] if square else other[i])
+        assert t[i] == want, (i, hex(t[i] ^ want))

@@ -49,9 +49,16 @@ out["encrypt_keyholder_tc_per_s"] = count / t
 os.environ["FLB_TC"] = "0"
 t = timed(lambda: flb.encrypt(pub, m, seed=3), reps=1)
 out["encrypt_public_per_s"] = count / t
-t = timed(lambda: flb.decrypt(priv, c))
-out["decrypt_per_s"] = count / t
-d = flb.decrypt(priv, c)
-out["roundtrip_ok"] = bool(torch.equal(d, m))
+for tc in ("0", "1"):
+    os.environ["FLB_TC"] = tc
+    sfx = "_tc" if tc == "1" else ""
+    t = timed(lambda: flb.decrypt(priv, c))
+    out["decrypt%s_per_s" % sfx] = count / t
+    c2 = c[:16645]
+    t = timed(lambda: flb.decrypt(priv, c2))
+    out["decrypt%s_16645_per_s" % sfx] = c2.shape[0] / t
+    d = flb.decrypt(priv, c)
+    out["roundtrip%s_ok" % sfx] = bool(torch.equal(d, m))
+os.environ["FLB_TC"] = "0"
 out["crt_equals_public"] = bool(torch.equal(c, flb.encrypt(pub, m, seed=3)))
 print(json.dumps(out))

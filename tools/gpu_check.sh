@@ -16,7 +16,8 @@ if [ "${NCU:-1}" = "1" ]; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
     --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e \
     > gpurun_out/${TAG}_bench_under_ncu.log 2>&1
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"k_encrypt" -c 2 \
+  # the tensor-core kernels of the step: key-holder stage 1 (k_tc_exp<32>), stage 2 and decryption (k_tc_exp<64>)
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"${NCU_K:-k_tc_exp}" -c ${NCU_C:-3} \
     -o gpurun_out/${TAG}_prof_enc python tools/prof_c2.py > gpurun_out/${TAG}_ncu_full.log 2>&1
 fi
 cat gpurun_out/${TAG}_pytest_gpu.txt gpurun_out/${TAG}_smoke.txt
