@@ -375,6 +375,7 @@ def run_flb(args):
         try:
             enc_tc = flb.op_cost(priv, "encrypt_crt_tc")
             dec_tc = flb.op_cost(priv, "decrypt_tc")
+            enc_macs = flb.op_cost(priv, "encrypt_crt_tc_macs")[1]
         except flb.FlbError:
             enc_tc = dec_tc = None
     if args.encrypt == "keyholder":
@@ -399,9 +400,9 @@ def run_flb(args):
         # IMAD-pipe work the tensor-core kernels actually issue: S^2 per Montgomery product
         imad_lp = enc_tc[1]
         achieved = imad_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12
-        per_unit = {"mont_muls": enc_tc[0], "imad_limb_products": imad_lp, "u8_macs": 32 * imad_lp,
+        per_unit = {"mont_muls": enc_tc[0], "imad_limb_products": imad_lp, "u8_macs": enc_macs,
                     "cios_equivalent_limb_products": enc_lp}
-        tensor = {"achieved": 32 * imad_lp * enc_units / (phase["t_enc"] * 1e-3) / 1e12, "peak": mma_peak,
+        tensor = {"achieved": enc_macs * enc_units / (phase["t_enc"] * 1e-3) / 1e12, "peak": mma_peak,
                   "unit": "T u8 MAC/s (tcgen05.mma kind::i8)",
                   "peak_basis": "148 SM x 7.26K MAC/clk/SM (tools/tc_i8_probe.cu) x %.0f MHz" % sm_mhz_max}
         tensor["frac"] = tensor["achieved"] / mma_peak
@@ -733,6 +734,15 @@ def run_other(args):
             ms, ph = run_steps(step, names)
             lp = {k: flb.op_cost(priv if k in ("decrypt", "encrypt_crt") else pub, k)[1]
                   for k in ("encrypt", "encrypt_crt", "decrypt", "add")}
+            # tensor-core kernels: count the IMAD-pipe work they actually issue (op_cost 5/6)
+            acct = {"encrypt_crt": "cios", "decrypt": "cios"}
+            if os.environ.get("FLB_TC", "1") != "0":
+                for k, tk in (("encrypt_crt", "encrypt_crt_tc"), ("decrypt", "decrypt_tc")):
+                    try:
+                        lp[k] = flb.op_cost(priv, tk)[1]
+                        acct[k] = "tensor-core (IMAD-pipe limb products of t = a b; reduction on tcgen05)"
+                    except flb.FlbError:
+                        pass
             peak = 148 * PEAK_LP_PER_CLK_SM * 1965e6
             per[str(bits)] = {
                 "batch": M,
@@ -741,7 +751,8 @@ def run_other(args):
                 "frac_roofline": {"encrypt": lp["encrypt"] * M / (ph["enc"] * 1e-3) / peak,
                                   "encrypt_keyholder": lp["encrypt_crt"] * M / (ph["enc_crt"] * 1e-3) / peak,
                                   "decrypt": lp["decrypt"] * M / (ph["dec"] * 1e-3) / peak,
-                                  "add": lp["add"] * M / (ph["add"] * 1e-3) / peak}}
+                                  "add": lp["add"] * M / (ph["add"] * 1e-3) / peak},
+                "imad_accounting": acct}
             del c, o, dm, m
         v = per["2048"]
         res.update(value=3.0 / (1 / v["encrypt_per_s"] + 1 / v["decrypt_per_s"] + 1 / v["add_per_s"]),

@@ -239,6 +239,20 @@ static uint64_t sched_mults(const H::Schedule& S) {
   return m;
 }
 
+static uint64_t sched_squarings(const H::Schedule& S) {
+  uint64_t q = (S.table > 1) ? 1u : 0u;  // x^2 of the table
+  for (size_t i = 1; i < S.ops.size(); i++) q += S.ops[i] & 0xffffu;
+  return q;
+}
+
+// IMAD-pipe limb products of the tensor-core kernel (flb_tc.cuh) for `mults` S-word Montgomery
+// products of which `sqr` are squarings: S^2 for the row-scan product, 10 (S/4)^2 for the block
+// squaring (FLB_TC_SQR, S >= 64)
+static uint64_t tc_imad_lp(uint64_t S, uint64_t mults, uint64_t sqr) {
+  const uint64_t sq_lp = (FLB_TC_SQR && S >= 64) ? 10 * (S / 4) * (S / 4) : S * S;
+  return (mults - sqr) * S * S + sqr * sq_lp;
+}
+
 int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls, uint64_t* limb_products) {
   if (!mont_muls || !limb_products) return fail(FLB_EINVAL, "null output");
   const flb_pub* P = K ? K : (V ? V->pub : nullptr);
@@ -287,16 +301,35 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       const uint64_t h = V->H;
       const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
       const uint64_t s2 = (1 + sched_mults(V->sched_p) + 2) + (1 + sched_mults(V->sched_q) + 2);
+      const uint64_t q12 = sched_squarings(V->sched_q) + sched_squarings(V->sched_p);  // same exponents
       *mont_muls = s1 + s2;
-      *limb_products = s1 * h * h + s2 * sp * sp;
+      *limb_products = tc_imad_lp(h, s1, q12) + tc_imad_lp(sp, s2, q12);
       return FLB_OK;
     }
     case 6: {  // decryption, tensor-core kernel (k_tc_exp) only: per prime 2 (entry) + table + schedule + 1
       if (!V || !V->tc) return fail(FLB_EUNSUPPORTED, "no tensor-core decryption path for this key");
-      uint64_t mm = 0;
-      for (int i = 0; i < 2; i++) mm += 2 + sched_mults(V->pr[i].sched) + 1;
+      uint64_t mm = 0, sq = 0;
+      for (int i = 0; i < 2; i++) {
+        mm += 2 + sched_mults(V->pr[i].sched) + 1;
+        sq += sched_squarings(V->pr[i].sched);
+      }
       *mont_muls = mm;
-      *limb_products = mm * sp * sp;
+      *limb_products = tc_imad_lp(sp, mm, sq);
+      return FLB_OK;
+    }
+    case 7:    // key-holder encryption, tensor-core kernels: *limb_products = u8 MACs (2 KB^2 per product)
+    case 8: {  // decryption exponentiations, tensor-core kernel: likewise
+      uint64_t mm, lp;
+      const int rc = flb_op_cost(K, V, op - 2, &mm, &lp);
+      if (rc) return rc;
+      if (op == 7) {
+        const uint64_t h = V->H;
+        const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
+        *limb_products = 32 * (s1 * h * h + (mm - s1) * sp * sp);
+      } else {
+        *limb_products = 32 * mm * sp * sp;
+      }
+      *mont_muls = mm;
       return FLB_OK;
     }
     case 2:

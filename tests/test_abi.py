@@ -161,3 +161,56 @@ def test_mod_create_and_rsa_keygen_host_logic():
     assert flb.rsa_keygen(512, 7) == (n, e, d, p, q)
     with pytest.raises(flb.FlbError):
         flb.rsa_keygen(100, 1)
+
+
+def _sliding_counts(e, w):
+    """(multiplications, of which squarings) of the odd-power sliding window, counted independently."""
+    bits = bin(e)[2:]
+    table = 1 << (w - 1)
+    mults, sq = (table, 1) if table > 1 else (0, 0)
+    i, first = 0, True
+    while i < len(bits):
+        if bits[i] == "0":
+            mults, sq, i = mults + 1, sq + 1, i + 1
+            continue
+        j = min(len(bits), i + w)
+        while bits[j - 1] == "0":
+            j -= 1
+        if not first:
+            mults, sq = mults + (j - i) + 1, sq + (j - i)
+        first = False
+        i = j
+    return mults, sq
+
+
+def test_op_cost_tensor_core_paths():
+    """Accounting of the tensor-core kernels (bench.py's roofline): Montgomery products per element,
+    IMAD-pipe limb products (S^2 per product, 10 (S/4)^2 per block squaring at S = 64) and u8 MACs
+    (2 (4S)^2 per product), against an independent window count."""
+    p, q = KEYS["2048"]
+    pub, priv = flb.key_from_primes(p, q)
+    sp, h = 64, 32
+
+    def best(e):
+        costs = [_sliding_counts(e, w) for w in range(1, 8)]
+        m = min(c[0] for c in costs)
+        return m, {c[1] for c in costs if c[0] == m}
+
+    mm, lp = flb.op_cost(priv, "decrypt_tc")
+    (mp, sqp), (mq, sqq) = best(p - 1), best(q - 1)
+    assert mm == mp + mq + 2 * 3
+    assert any(lp == (mm - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in sqp for b in sqq)
+    assert flb.op_cost(priv, "decrypt_tc_macs") == (mm, 32 * mm * sp * sp)
+    mm_e, lp_e = flb.op_cost(priv, "encrypt_crt_tc")
+    (ep, esp), (eq, esq) = best(p), best(q)
+    s1 = (2 + eq + 1) + (2 + ep + 1)      # stage 1: r^Q mod p, r^P mod q at the half frame
+    s2 = (1 + ep + 2) + (1 + eq + 2)      # stage 2: y^P mod P^2
+    assert mm_e == s1 + s2
+    assert any(lp_e == s1 * h * h + (s2 - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2
+               for a in esp for b in esq)
+    assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, 32 * (s1 * h * h + s2 * sp * sp))
+    # 1024-bit keys have no two-stage (half-frame) encryption path
+    p1, q1 = KEYS["1024"]
+    _, priv1 = flb.key_from_primes(p1, q1)
+    with pytest.raises(flb.FlbError):
+        flb.op_cost(priv1, "encrypt_crt_tc")
