@@ -14,9 +14,10 @@
 // Tile: 128 elements per CTA (MMA M = 128, one per TMEM lane), 256 threads, two CTAs per SM so the
 // warp schedulers overlap one CTA's product phase (integer pipe) with the other's normalisation
 // (ALU, TMEM loads, barriers).  Per multiplication (KB = 4S bytes per operand):
-//   P   two halves of 64 elements: groups of T = 4 lanes compute t = a b (row-scanning product,
-//       X = S/4 limbs per lane, the multiplier staged in the element's sA row); t_lo goes to sA as
-//       bytes (the MMA A operand), t_hi to the element's work row;
+//   P   groups of T lanes (X = S/T = 16 limbs each; T = 4 at S = 64 in two passes of 64 elements,
+//       T = 2 at S = 32 in one pass of 128) compute t = a b (row-scanning product, the multiplier
+//       staged in the element's sA row; squarings at S = 64 by block squaring, tc_square_product);
+//       t_lo goes to sA as bytes (the MMA A operand), t_hi to the element's work row;
 //   M1  one thread: D1[128 x KB] = sA x B1, B1[n][k] = N'_(n-k) (bytes, k <= n);
 //   N1  8 warps (TMEM lane quadrant w % 4, column half w / 4): q = D1 mod R normalised into bytes
 //       over sA, the carry between the column halves resolved exactly through shared memory;
@@ -36,12 +37,14 @@ namespace tc {
 
 constexpr int kTileM = 128;     // elements per CTA tile (MMA M, TMEM lanes)
 constexpr int kThreads = 256;   // 8 warps; two CTAs per SM
-constexpr int kHalf = 64;       // elements per product half-phase
-constexpr int kT = 4;           // lanes per element in the product phase
+constexpr int kT = 4;           // lanes per element in the product phase at S >= 64 (S = 32: 2)
 
 template <int S>
 struct Cfg {
-  static constexpr int X = S / kT;                 // limbs per lane
+  static constexpr int T = S >= 64 ? kT : 2;       // lanes per element in the product phase
+  static constexpr int X = S / T;                  // limbs per lane (16)
+  static constexpr int EP = kThreads / T;          // elements per product pass
+  static constexpr int NP = kTileM / EP;           // product passes per tile
   static constexpr int KB = 4 * S;                 // bytes of an S-word operand (MMA K and N)
   static constexpr int KCH = KB / 16;              // 16-byte chunks per operand row
   static constexpr int QW = S / 2, QC = KB / 2;    // words / byte columns per normalising thread
@@ -177,7 +180,7 @@ static __device__ unsigned long long g_tc_prof[8];
 template <int S>
 __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s, int elem, const uint32_t* sW) {
   using C = Cfg<S>;
-  const int k = threadIdx.x % kT;
+  const int k = threadIdx.x % C::T;
   if (s.row) {
     const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + k * C::X);
 #pragma unroll
@@ -186,7 +189,7 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
       r[4 * v] = u.x; r[4 * v + 1] = u.y; r[4 * v + 2] = u.z; r[4 * v + 3] = u.w;
     }
   } else {
-    load_elem<C::X, kT>(r, s.p + (size_t)elem * s.stride, s.words, (uint32_t)elem < s.valid);
+    load_elem<C::X, C::T>(r, s.p + (size_t)elem * s.stride, s.words, (uint32_t)elem < s.valid);
   }
 }
 
@@ -329,23 +332,154 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
     *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
 }
 
+// Block squaring with the pieces summed in registers (FLB_TC_SQR == 2): the same block products as
+// tc_square_product, but each lane accumulates its own quarter Q_k = t[2Xk, 2Xk + 2X) in registers,
+// the off-diagonal pieces (undoubled) arriving from the lanes that computed them by shuffle; the
+// diagonal block a_k^2 is folded in last as t_k = 2 acc + a_k^2, and the quarters' carries are
+// resolved by one shuffle round plus a ballot carry-lookahead.  Shared memory sees only the final
+// quarter stores (no read-modify-write of t).
+template <int S>
+__device__ __forceinline__ void tc_square_product_reg(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
+                                                      uint32_t* sW) {
+  constexpr int X = Cfg<S>::X, H = X / 2, Q = 2 * X;
+  const int k = threadIdx.x % kT;
+  uint32_t acc[Q];
+  uint32_t qc = 0;  // carries out of the quarter (weight 2^(32 Q)), of the undoubled off-diagonal sum
+  {
+    // half block of lane k: a_i a_(i+2)[H hh, + H), i = k & 1, hh = k >> 1, at words Q i + Q + H hh:
+    // lane 0 -> Q_1 [0, X + H), lane 2 -> Q_1 [H, Q), lane 1 -> Q_2 [0, X + H), lane 3 -> Q_2 [H, Q)
+    uint32_t v[X + H];
+    {
+      uint32_t M[X];
+      const int i = k & 1, hh = k >> 1;
+#pragma unroll
+      for (int j = 0; j < X; j++) M[j] = __shfl_sync(FULL, a[j], i, kT);
+      blk_prod<X, H>(v, M, a, i + 2, hh == 1);
+    }
+    const bool rcv = (k == 1 || k == 2);
+#pragma unroll
+    for (int w = 0; w < X + H; w++) {
+      const uint32_t x = __shfl_up_sync(FULL, v[w], 1, kT);  // lane 1 <- lane 0, lane 2 <- lane 1
+      acc[w] = rcv ? x : 0u;
+    }
+#pragma unroll
+    for (int w = X + H; w < Q; w++) acc[w] = 0;
+    uint64_t cy = 0;
+#pragma unroll
+    for (int w = 0; w < X + H; w++) {
+      const uint32_t y = __shfl_down_sync(FULL, v[w], 1, kT);  // lane 1 <- lane 2, lane 2 <- lane 3
+      const uint64_t s = (uint64_t)acc[H + w] + (rcv ? y : 0u) + cy;
+      acc[H + w] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    qc += (uint32_t)cy;
+  }
+  {
+    // full block F_k = a_k a_(k+1 mod 4) at words X (2k + 1) (lane 3: 3X): low half -> Q_k [X, Q)
+    // (lane 3's -> Q_1), high half -> Q_(k+1) [0, X) (lane 3's -> Q_2)
+    uint32_t v[Q];
+    blk_prod<X, X>(v, a, a, (k + 1) & (kT - 1), false);
+    uint64_t cy = 0;
+#pragma unroll
+    for (int j = 0; j < X; j++) {
+      const uint32_t r3 = __shfl_sync(FULL, v[j], kT - 1, kT);
+      const uint64_t s = (uint64_t)acc[X + j] + (k < kT - 1 ? v[j] : 0u) + (k == 1 ? r3 : 0u) + cy;
+      acc[X + j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    qc += (uint32_t)cy;
+    cy = 0;
+#pragma unroll
+    for (int j = 0; j < X; j++) {
+      const uint32_t u = __shfl_up_sync(FULL, v[X + j], 1, kT);
+      const uint32_t r3 = __shfl_sync(FULL, v[X + j], kT - 1, kT);
+      const uint64_t s = (uint64_t)acc[j] + (k >= 1 ? u : 0u) + (k == 2 ? r3 : 0u) + cy;
+      acc[j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+#pragma unroll
+    for (int j = X; j < Q; j++) {
+      const uint64_t s = (uint64_t)acc[j] + cy;
+      acc[j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    qc += (uint32_t)cy;
+  }
+  uint32_t cq;
+  {
+    // diagonal: Q_k = 2 acc + a_k^2, the product's low words folded in as its rows emerge
+    uint32_t E[X + 1], O[X + 1], pend = 0;
+#pragma unroll
+    for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
+    uint64_t cy = 0;
+    uint32_t prev = 0;
+#pragma unroll
+    for (int j = 0; j < X; j++) {
+      const uint32_t o = local_row<X>(E, O, pend, a, a[j]);
+      const uint32_t d = (acc[j] << 1) | (prev >> 31);
+      prev = acc[j];
+      const uint64_t s = (uint64_t)d + o + cy;
+      acc[j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    uint32_t hw[X];
+    asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(hw[0]) : "r"(E[0]), "r"(pend));
+#pragma unroll
+    for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(hw[t]) : "r"(E[t]), "r"(O[t - 1]));
+#pragma unroll
+    for (int t = 0; t < X; t++) {
+      const uint32_t d = (acc[X + t] << 1) | (prev >> 31);
+      prev = acc[X + t];
+      const uint64_t s = (uint64_t)d + hw[t] + cy;
+      acc[X + t] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    cq = 2 * qc + (prev >> 31) + (uint32_t)cy;
+  }
+  // carries between quarters: Q_(k-1)'s carry-out into Q_k, then single-bit ripples by lookahead
+  {
+    uint32_t cin = __shfl_up_sync(FULL, cq, 1, kT);
+    if (k == 0) cin = 0;
+    uint64_t cy = cin;
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+      const uint64_t s = (uint64_t)acc[j] + cy;
+      acc[j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+    const uint32_t c = group_carry<kT>(cy != 0, all_ones<Q>(acc), 0);
+    add_word_propagate<Q>(acc, c & 1u);
+  }
+#pragma unroll
+  for (int c = 0; c < X / 2; c++)
+    *t_chunk<S>(sA, sW, elem, Q * k + 4 * c) = make_uint4(acc[4 * c], acc[4 * c + 1], acc[4 * c + 2], acc[4 * c + 3]);
+}
+
 // The product phase of tc_mont: t = a b (2S words) for the 128 elements of the tile, t_lo into the
-// elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of kT lanes per element,
-// two halves of 64 elements.  CTA-collective (no trailing barrier).
+// elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of T lanes per element
+// (X = 16 limbs each), NP passes of EP elements.  CTA-collective (no trailing barrier).
 template <int S>
 __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq, uint8_t* sA, uint32_t* sW) {
   using C = Cfg<S>;
   constexpr int X = C::X, KCH = C::KCH;
-  const int tid = threadIdx.x, k = tid % kT;
-  // ---- P: t = a b, two halves of 64 elements
+  constexpr int T = C::T;
+  const int tid = threadIdx.x, k = tid % T;
+  // ---- P: t = a b, NP passes of EP elements (S = 64: two passes of 64; S = 32: one of 128)
 #pragma unroll 1
-  for (int h = 0; h < 2; h++) {
-    const int elem = h * kHalf + tid / kT;
+  for (int h = 0; h < C::NP; h++) {
+    const int elem = h * C::EP + tid / T;
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
-    if (FLB_TC_SQR && S >= 64 && sq) {  // measured: a gain at S = 64, a loss at S = 32
-      tc_square_product<S>(a, elem, sA, sW);
-      continue;
+    if constexpr (FLB_TC_SQR && S >= 64) {  // block squaring needs X x X blocks on 4 lanes
+      if (sq) {
+        if (FLB_TC_SQR == 2) {
+          __syncwarp();  // a may come from the work row the quarters are stored into
+          tc_square_product_reg<S>(a, elem, sA, sW);
+        } else {
+          tc_square_product<S>(a, elem, sA, sW);
+        }
+        continue;
+      }
     }
     if (sq) {
 #pragma unroll
@@ -367,19 +501,19 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
 #pragma unroll
     for (int t = 0; t < X; t++) lo[t] = 0;
 #pragma unroll 1
-    for (int kk = 0; kk < kT; kk++) {
+    for (int kk = 0; kk < T; kk++) {
 #pragma unroll
       for (int j4 = 0; j4 < X; j4 += 4) {
         const uint4 bq = *reinterpret_cast<const uint4*>(sA + cm_off(elem, 4u * (kk * X + j4), KCH));
         const uint32_t bw[4] = {bq.x, bq.y, bq.z, bq.w};
 #pragma unroll
         for (int u = 0; u < 4; u++) {
-          const uint32_t o = cios_step<X, kT, false>(E, O, pend, a, bw[u], dummy, 0u);
+          const uint32_t o = cios_step<X, T, false>(E, O, pend, a, bw[u], dummy, 0u);
           if (k == kk) lo[j4 + u] = o;
         }
       }
     }
-    collapse<X, kT>(hi, E, O, pend);
+    collapse<X, T>(hi, E, O, pend);
     __syncwarp();
 #pragma unroll
     for (int v = 0; v < X / 4; v++) {
@@ -398,7 +532,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
                                         const uint32_t* __restrict__ Nmod, uint32_t& phase) {
   using C = Cfg<S>;
   constexpr int X = C::X, KCH = C::KCH, KB = C::KB, QW = C::QW, QC = C::QC;
-  const int tid = threadIdx.x, k = tid % kT, warp = tid >> 5;
+  const int tid = threadIdx.x, warp = tid >> 5;
   uint8_t* sA = sm.base + C::OFF_A;
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
 #if FLB_TC_PROF
@@ -601,10 +735,10 @@ template <int S>
 __device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint32_t stride, uint32_t valid) {
   using C = Cfg<S>;
   const uint32_t* sW = reinterpret_cast<const uint32_t*>(sm.base + C::OFF_W);
-  const int k = threadIdx.x % kT;
+  const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < 2; h++) {
-    const int elem = h * kHalf + threadIdx.x / kT;
+  for (int h = 0; h < C::NP; h++) {
+    const int elem = h * C::EP + threadIdx.x / C::T;
     if ((uint32_t)elem < valid) {
       const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + k * C::X);
       uint4* o = reinterpret_cast<uint4*>(dst + (size_t)elem * stride + k * C::X);
@@ -620,15 +754,15 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
   using C = Cfg<S>;
   constexpr int X = C::X;
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
-  const int k = threadIdx.x % kT;
+  const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < 2; h++) {
-    const int elem = h * kHalf + threadIdx.x / kT;
+  for (int h = 0; h < C::NP; h++) {
+    const int elem = h * C::EP + threadIdx.x / C::T;
     uint32_t r[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
-    load_const<X, kT>(nn, Nmod);
-    grp_add_small<X, kT>(r, 1u);
-    grp_cond_sub<X, kT>(r, nn, 0u);
+    load_const<X, C::T>(nn, Nmod);
+    grp_add_small<X, C::T>(r, 1u);
+    grp_cond_sub<X, C::T>(r, nn, 0u);
     uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + k * X);
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
@@ -642,16 +776,16 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
   using C = Cfg<S>;
   constexpr int X = C::X;
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
-  const int k = threadIdx.x % kT;
+  const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < 2; h++) {
-    const int elem = h * kHalf + threadIdx.x / kT;
+  for (int h = 0; h < C::NP; h++) {
+    const int elem = h * C::EP + threadIdx.x / C::T;
     uint32_t r[X], a[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
     src_load<S>(a, s, elem, sW);
-    load_const<X, kT>(nn, Nmod);
-    const uint32_t cy = grp_add<X, kT>(r, r, a);
-    grp_cond_sub<X, kT>(r, nn, cy);
+    load_const<X, C::T>(nn, Nmod);
+    const uint32_t cy = grp_add<X, C::T>(r, r, a);
+    grp_cond_sub<X, C::T>(r, nn, cy);
     uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + k * X);
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
