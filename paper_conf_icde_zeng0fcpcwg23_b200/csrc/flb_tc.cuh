@@ -196,6 +196,9 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
 #ifndef FLB_TC_SQR
 #define FLB_TC_SQR 1  // block squaring in the product phase (0: squarings use the general product)
 #endif
+#ifndef FLB_TC_SQR32
+#define FLB_TC_SQR32 1  // block squaring also at S = 32 (two lanes per element)
+#endif
 
 // ----------------------------------------------------------------------------- squaring product
 // t = a^2 for the product phase when a = b (87 % of the multiplications of a modexp).  Lane k of the
@@ -208,7 +211,7 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
 // are accumulated in place in t's destination rows (t_lo: the element's sA row, the MMA operand;
 // t_hi: its work row) in phases with disjoint word ranges, their carry-outs folded in by one final
 // group pass with a ballot carry-lookahead.
-template <int X, int R>
+template <int X, int R, int W = kT>
 __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t (&M)[X], const uint32_t (&a)[X],
                                          int src, bool own_upper) {
   // out = M x (R row words of lane src's block): words [0, R) of it by shuffle (every lane serves its
@@ -218,7 +221,7 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
   for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
 #pragma unroll
   for (int j = 0; j < R; j++) {
-    uint32_t bj = __shfl_sync(FULL, a[j], src, kT);
+    uint32_t bj = __shfl_sync(FULL, a[j], src, W);
     if (R < X && own_upper) bj = a[(j + R) % X];
     out[j] = local_row<X>(E, O, pend, M, bj);
   }
@@ -330,6 +333,59 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
 #pragma unroll
   for (int cc = 0; cc < X / 2; cc++)
     *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
+}
+
+// Block squaring for two lanes per element (S = 32, X = 16): lane k computes a_k^2 (X x X, stored to
+// t[2Xk, 2Xk + 2X)) and half of the cross block, a_0 a_1[H k, + H) (X x H, doubled, added at words
+// X + H k), 384 instead of 512 limb products per lane.  The two cross pieces overlap, so they are
+// added in two phases; both carries land in lane 1's half and are folded in by lane 1.
+template <int S>
+__device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
+                                                     uint32_t* sW) {
+  constexpr int X = Cfg<S>::X, H = X / 2;
+  const int k = threadIdx.x % 2;
+  {
+    uint32_t v[2 * X];
+    blk_prod<X, X, 2>(v, a, a, k, false);
+    __syncwarp();  // both lanes have read a (it may come from the work row)
+#pragma unroll
+    for (int c = 0; c < X / 2; c++)
+      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  }
+  uint32_t cx = 0;
+  {
+    uint32_t M[X], v[X + H];
+#pragma unroll
+    for (int j = 0; j < X; j++) M[j] = __shfl_sync(FULL, a[j], 0, 2);
+    // rows [0, H) of a_1 come from lane 1 (read by lane 0); lane 1 takes its own rows [H, X)
+    blk_prod<X, H, 2>(v, M, a, 1, k == 1);
+    __syncwarp();
+    if (k == 0) cx = t_add_dbl<S, X + H>(sA, sW, elem, X, v);      // [X, 2X + H): carry at 2X + H
+    __syncwarp();
+    if (k == 1) cx = t_add_dbl<S, X + H>(sA, sW, elem, X + H, v);  // [X + H, 3X): carry at 3X
+    __syncwarp();
+  }
+  const uint32_t c0 = __shfl_sync(FULL, cx, 0, 2);
+  if (k == 1) {
+    // lane 1's half t[2X, 4X): + c0 at relative H, + cx at relative X (no carry leaves t)
+    uint32_t q[2 * X];
+#pragma unroll
+    for (int c = 0; c < X / 2; c++) {
+      const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X + 4 * c);
+      q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
+    }
+    uint64_t cy = 0;
+#pragma unroll
+    for (int j = H; j < 2 * X; j++) {
+      const uint64_t s = (uint64_t)q[j] + (j == H ? c0 : 0u) + (j == X ? cx : 0u) + cy;
+      q[j] = (uint32_t)s;
+      cy = s >> 32;
+    }
+#pragma unroll
+    for (int c = H / 4; c < X / 2; c++)
+      *t_chunk<S>(sA, sW, elem, 2 * X + 4 * c) = make_uint4(q[4 * c], q[4 * c + 1], q[4 * c + 2], q[4 * c + 3]);
+  }
+  __syncwarp();
 }
 
 // Block squaring with the pieces summed in registers (FLB_TC_SQR == 2): the same block products as
@@ -470,6 +526,14 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
     const int elem = h * C::EP + tid / T;
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
+#if FLB_TC_SQR32
+    if constexpr (FLB_TC_SQR && T == 2) {
+      if (sq) {
+        tc_square_product_t2<S>(a, elem, sA, sW);
+        continue;
+      }
+    }
+#endif
     if constexpr (FLB_TC_SQR && S >= 64) {  // block squaring needs X x X blocks on 4 lanes
       if (sq) {
         if (FLB_TC_SQR == 2) {

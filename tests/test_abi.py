@@ -185,7 +185,8 @@ def _sliding_counts(e, w):
 
 def test_op_cost_tensor_core_paths():
     """Accounting of the tensor-core kernels (bench.py's roofline): Montgomery products per element,
-    IMAD-pipe limb products (S^2 per product, 10 (S/4)^2 per block squaring at S = 64) and u8 MACs
+    IMAD-pipe limb products (S^2 per product; block squaring 10 (S/4)^2 at S = 64, 3 (S/2)^2 at
+    S = 32) and u8 MACs
     (2 (4S)^2 per product), against an independent window count."""
     p, q = KEYS["2048"]
     pub, priv = flb.key_from_primes(p, q)
@@ -206,8 +207,9 @@ def test_op_cost_tensor_core_paths():
     s1 = (2 + eq + 1) + (2 + ep + 1)      # stage 1: r^Q mod p, r^P mod q at the half frame
     s2 = (1 + ep + 2) + (1 + eq + 2)      # stage 2: y^P mod P^2
     assert mm_e == s1 + s2
-    assert any(lp_e == s1 * h * h + (s2 - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2
-               for a in esp for b in esq)
+    # stage 1 (h = 32 words, two lanes): squarings 3 (h/2)^2; stage 2 (64 words, four lanes): 10 (sp/4)^2
+    assert any(lp_e == (s1 - a - b) * h * h + (a + b) * 3 * (h // 2) ** 2
+               + (s2 - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in esp for b in esq)
     assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, 32 * (s1 * h * h + s2 * sp * sp))
     # 1024-bit keys have no two-stage (half-frame) encryption path
     p1, q1 = KEYS["1024"]
