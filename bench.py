@@ -524,7 +524,8 @@ def run_flb(args):
                          "frac": achieved / peak, "traffic": traffic, "per_unit": per_unit,
                          "peak_basis": "148 SM x 32 IMAD.WIDE/clk/SM x %.0f MHz (guide: IMAD rt=2/SMSP; "
                                        "IMAD.WIDE half rate, measured tools/imad_peak.cu)" % sm_mhz_max,
-                         "tensor": tensor, "cios_equivalent_achieved": cios_eq},
+                         "tensor": tensor, "cios_equivalent_achieved": cios_eq,
+                         "cios_equivalent_frac": cios_eq / peak},
             "decrypt_cost": {"mont_muls": dec_mm, "limb_products": dec_lp},
             "decrypt_roofline": dec_roof,
             "clocks": clk, "gpu_launches": launches_per_step * args.steps,
