@@ -370,6 +370,7 @@ def run_flb(args):
 
     # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
     tc_on = os.environ.get("FLB_TC", "1") != "0"
+    dag_on = os.environ.get("FLB_TC_DAG", "1") != "0" and KEY_BITS == 2048
     enc_tc = dec_tc = None
     if tc_on:
         try:
@@ -380,7 +381,10 @@ def run_flb(args):
             enc_tc = dec_tc = None
     if args.encrypt == "keyholder":
         enc_mm, enc_lp = flb.op_cost(priv, "encrypt_crt")
-        if enc_tc:
+        if enc_tc and dag_on:
+            enc_kernel = ("k_tc_exp_dag<32,64> (both key-holder stages in one launch, stage-2 tiles wait on their "
+                          "stage-1 tile; Montgomery reduction as u8 tcgen05 MMAs, t = a b on the IMAD pipe)")
+        elif enc_tc:
             enc_kernel = ("k_tc_exp<32> + k_tc_exp<64> (two-stage key-holder encryption; Montgomery reduction as "
                           "u8 tcgen05 MMAs, t = a b on the IMAD pipe)")
         else:
@@ -493,10 +497,10 @@ def run_flb(args):
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": r["sample"],
                "per_op_seconds": {"encrypt": r["t_enc"], "decrypt": r["t_dec"], "add": r["t_add"]}}
 
-    # pack per client; encrypt (TC: Philox fill, k_tc_exp<32>, k_tc_exp<64>, k_crt_combine; CIOS:
-    # k_crt_pre, k_encrypt_crt2); reduce (plan scan, plan fill, k_reduce); exchange + finish (N > 1);
-    # decrypt (TC: k_tc_exp<64>, k_dec_finish; CIOS: k_decrypt); unpack
-    enc_launches = (4 if enc_tc else 2) if args.encrypt == "keyholder" else 1
+    # pack per client; encrypt (TC: Philox fill, k_tc_exp_dag (or k_tc_exp<32>, k_tc_exp<64>),
+    # k_crt_combine; CIOS: k_crt_pre, k_encrypt_crt2); reduce (plan scan, plan fill, k_reduce);
+    # exchange + finish (N > 1); decrypt (TC: k_tc_exp<64>, k_dec_finish; CIOS: k_decrypt); unpack
+    enc_launches = ((3 if dag_on else 4) if enc_tc else 2) if args.encrypt == "keyholder" else 1
     launches_per_step = (CLIENTS + enc_launches + 3 + (3 if world > 1 else 0) + (2 if dec_tc else 1)
                          + (1 if my_values else 0))
     if rank == 0:

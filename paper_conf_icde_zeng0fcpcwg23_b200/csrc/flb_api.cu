@@ -434,6 +434,11 @@ static bool tc_enabled() {
   const char* e = getenv("FLB_TC");
   return !(e && atoi(e) == 0);
 }
+// FLB_TC_DAG=0: the two key-holder stages as two k_tc_exp launches instead of one k_tc_exp_dag
+static bool tc_dag_enabled() {
+  const char* e = getenv("FLB_TC_DAG");
+  return !(e && atoi(e) == 0);
+}
 static bool use_tc(const flb_priv* V) { return V->tc && tc_enabled(); }
 static bool use_tc_half(const flb_priv* V) { return V->tc_half && tc_enabled(); }
 
@@ -740,6 +745,8 @@ static int crt2_dispatch(const flb_priv* V, const uint32_t* dev, const uint32_t*
 
 static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
                           uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  if (use_tc(V) && use_tc_half(V) && V->H == 32 && V->pub->sp == 64 && tc_dag_enabled())
+    return run_encrypt_kh_dag<32, 64>(V, dev, m, r, seed, ctr0, c, count, st);  // 2048-bit keys: one launch
   Scratch ys;
   int rc = ys.alloc((size_t)2 * count * V->H * 4, st);
   if (rc) return rc;

@@ -499,40 +499,102 @@ int run_encrypt_crt2(const flb_priv* V, const uint32_t* dev, const uint32_t* m, 
 // ----------------------------------------------------------------------------- tensor-core modexp
 // One k_tc_exp launch over the (up to two) problems of A: persistent grid of two 256-thread CTAs
 // per SM (flb_tc.cuh), window-table scratch sized for the largest table.
-template <int S>
-int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
-  using C = flb::tc::Cfg<S>;
-  int dev_id = 0, sms = 0;
+template <typename F>
+int tc_set_attrs(F* kern, int smem_bytes) {
+  int dev_id = 0;
   FLB_CK(cudaGetDevice(&dev_id));
-  {
-    static std::mutex mu;
-    static std::map<int, bool> attr_done;  // function attributes are per device
-    std::lock_guard<std::mutex> lk(mu);
-    if (!attr_done[dev_id]) {
-      FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_exp<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-      FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_exp<S>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-      attr_done[dev_id] = true;
-    }
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, bool> done;  // function attributes are per device
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair((const void*)kern, dev_id);
+  if (!done[key]) {
+    FLB_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes));
+    FLB_CK(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+    done[key] = true;
   }
-  FLB_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id));
-  uint64_t tiles = 0;
-  int table = 1;
+  return FLB_OK;
+}
+
+// tile counts of A's problems; total tiles and the largest window table
+inline int tc_tiles(flb::tc::ExpArgs& A, uint64_t* tiles, int* table) {
+  *tiles = 0;
+  *table = 1;
   for (int i = 0; i < A.nprob; i++) {
     auto& P = A.pb[i];
     if (P.sched_len < 2) return fail(FLB_EUNSUPPORTED, "tensor-core path needs a multi-window exponent");
     P.tiles = (P.count + flb::tc::kTileM - 1) / flb::tc::kTileM;
-    tiles += P.tiles;
-    table = std::max(table, P.table);
+    *tiles += P.tiles;
+    *table = std::max(*table, P.table);
   }
   if (A.nprob < 2) A.pb[1].tiles = 0;
+  return FLB_OK;
+}
+
+inline int sm_count(int* sms) {
+  int dev_id = 0;
+  FLB_CK(cudaGetDevice(&dev_id));
+  FLB_CK(cudaDeviceGetAttribute(sms, cudaDevAttrMultiProcessorCount, dev_id));
+  return FLB_OK;
+}
+
+template <int S>
+int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
+  using C = flb::tc::Cfg<S>;
+  int rc = tc_set_attrs(flb::tc::k_tc_exp<S>, C::SMEM);
+  if (rc) return rc;
+  int sms = 0;
+  rc = sm_count(&sms);
+  if (rc) return rc;
+  uint64_t tiles = 0;
+  int table = 1;
+  rc = tc_tiles(A, &tiles, &table);
+  if (rc) return rc;
   if (tiles == 0) return FLB_OK;
   const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), tiles);  // two CTAs per SM
   Scratch s_tab;
-  int rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
+  rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
   if (rc) return rc;
   A.scratch = (uint32_t*)s_tab.p;
   A.tab_entries = table + 1;
   flb::tc::k_tc_exp<S><<<grid, flb::tc::kThreads, C::SMEM, st>>>(A);
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+// both key-holder stages in one k_tc_exp_dag launch (stage-1 problems A1 at S1 words, stage-2 problems
+// A2 at S2 words, the same element counts)
+template <int S1, int S2>
+int launch_tc_exp_dag(flb::tc::ExpArgs& A1, flb::tc::ExpArgs& A2, cudaStream_t st) {
+  constexpr int SMEM = flb::tc::Cfg<S1>::SMEM > flb::tc::Cfg<S2>::SMEM ? flb::tc::Cfg<S1>::SMEM
+                                                                       : flb::tc::Cfg<S2>::SMEM;
+  int rc = tc_set_attrs(flb::tc::k_tc_exp_dag<S1, S2>, SMEM);
+  if (rc) return rc;
+  int sms = 0;
+  rc = sm_count(&sms);
+  if (rc) return rc;
+  uint64_t t1 = 0, t2 = 0;
+  int tab1 = 1, tab2 = 1;
+  rc = tc_tiles(A1, &t1, &tab1);
+  if (rc) return rc;
+  rc = tc_tiles(A2, &t2, &tab2);
+  if (rc) return rc;
+  if (A1.nprob != 2 || A2.nprob != 2 || A1.pb[0].tiles != A2.pb[0].tiles || A1.pb[1].tiles != A2.pb[1].tiles)
+    return fail(FLB_EINVAL, "dag launch: the two stages must have the same problems' tile counts");
+  if (t1 == 0) return FLB_OK;
+  if (t1 >= 0xFFFFFFF0ull / 2) return fail(FLB_EINVAL, "dag launch: too many tiles");
+  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), t1 + t2);
+  const uint64_t stride = (uint64_t)flb::tc::kTileM * std::max<uint64_t>((uint64_t)(tab1 + 1) * S1,
+                                                                          (uint64_t)(tab2 + 1) * S2);
+  Scratch s_tab, s_sync;
+  rc = s_tab.alloc((size_t)grid * stride * 4, st);
+  if (rc) return rc;
+  rc = s_sync.alloc((size_t)(1 + t1) * 4, st);
+  if (rc) return rc;
+  FLB_CK(cudaMemsetAsync(s_sync.p, 0, (size_t)(1 + t1) * 4, st));
+  A1.scratch = A2.scratch = (uint32_t*)s_tab.p;
+  A1.tab_entries = tab1 + 1;
+  A2.tab_entries = tab2 + 1;
+  flb::tc::k_tc_exp_dag<S1, S2><<<grid, flb::tc::kThreads, SMEM, st>>>(A1, A2, (uint32_t*)s_sync.p, stride);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }
@@ -549,14 +611,11 @@ int run_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint
 
 // key-holder stage 2 on the tensor cores: c_P = (1 + m n) y_P^P mod P^2 for both primes in one
 // k_tc_exp launch, then k_crt_combine
+// stage-2 problems: c_P = (1 + m n) y_P^P mod P^2 for both primes (y = [2][count][H], out cpq [2][count][S])
 template <int S>
-int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
-                       size_t count, cudaStream_t st) {
-  Scratch s_out;
-  int rc = s_out.alloc((size_t)2 * count * S * 4, st);
-  if (rc) return rc;
-  uint32_t* cpq = (uint32_t*)s_out.p;
-  flb::tc::ExpArgs A{};
+void tc_stage2_args(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* cpq,
+                    size_t count, flb::tc::ExpArgs& A) {
+  A = flb::tc::ExpArgs{};
   A.nprob = 2;
   A.one = dev + V->o_one;
   for (int i = 0; i < 2; i++) {
@@ -579,11 +638,15 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
     P.out = cpq + (size_t)i * count * S;
     P.count = count;
   }
-  rc = launch_tc_exp<S>(A, st);
-  if (rc) return rc;
+}
+
+// c = CRT(c_p, c_q) for the key-holder encryption (k_crt_combine)
+template <int S>
+int tc_combine(const flb_priv* V, const uint32_t* dev, const uint32_t* cpq, uint32_t* c, size_t count,
+               cudaStream_t st) {
   constexpr int XC = 16, TC = S / 16;
   int cgrid;
-  rc = grid_for<TC>(flb::k_crt_combine<XC, TC>, count, &cgrid);
+  int rc = grid_for<TC>(flb::k_crt_combine<XC, TC>, count, &cgrid);
   if (rc) return rc;
   flb::CombineArgs B;
   B.P2 = {dev + V->pr[0].o_P2, V->pr[0].P2_n0inv};
@@ -598,13 +661,28 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
   return FLB_OK;
 }
 
+// key-holder stage 2 on the tensor cores: c_P = (1 + m n) y_P^P mod P^2 for both primes in one
+// k_tc_exp launch, then k_crt_combine
+template <int S>
+int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* y, uint32_t* c,
+                       size_t count, cudaStream_t st) {
+  Scratch s_out;
+  int rc = s_out.alloc((size_t)2 * count * S * 4, st);
+  if (rc) return rc;
+  uint32_t* cpq = (uint32_t*)s_out.p;
+  flb::tc::ExpArgs A;
+  tc_stage2_args<S>(V, dev, m, y, cpq, count, A);
+  rc = launch_tc_exp<S>(A, st);
+  if (rc) return rc;
+  return tc_combine<S>(V, dev, cpq, c, count, st);
+}
+
 // key-holder stage 1 on the tensor cores: y_P = r^Q mod P in the H-word frame (both primes, one
 // launch); r drawn by k_philox_fill unless the caller passes it
 template <int HS>
-int run_crt_pre_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0,
-                   uint32_t* y, size_t count, cudaStream_t st) {
+int tc_stage1_args(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0,
+                   uint32_t* y, size_t count, cudaStream_t st, Scratch& s_r, flb::tc::ExpArgs& A) {
   const uint32_t sp = V->pub->sp;
-  Scratch s_r;
   if (!r) {
     int rc = s_r.alloc((size_t)count * sp * 4, st);
     if (rc) return rc;
@@ -626,7 +704,7 @@ int run_crt_pre_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* r, ui
     FLB_LAUNCH_CHECK();
     r = (const uint32_t*)s_r.p;
   }
-  flb::tc::ExpArgs A{};
+  A = flb::tc::ExpArgs{};
   A.nprob = 2;
   A.one = dev + V->o_one;
   for (int i = 0; i < 2; i++) {
@@ -647,7 +725,36 @@ int run_crt_pre_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* r, ui
     P.out = y + (size_t)i * count * HS;
     P.count = count;
   }
+  return FLB_OK;
+}
+
+template <int HS>
+int run_crt_pre_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* r, uint64_t seed, uint64_t ctr0,
+                   uint32_t* y, size_t count, cudaStream_t st) {
+  Scratch s_r;
+  flb::tc::ExpArgs A;
+  int rc = tc_stage1_args<HS>(V, dev, r, seed, ctr0, y, count, st, s_r, A);
+  if (rc) return rc;
   return launch_tc_exp<HS>(A, st);
+}
+
+// both key-holder stages in one dependency-ordered launch (k_tc_exp_dag), then k_crt_combine:
+// y_P = r^Q mod P (HS words), c_P = (1 + m n) y_P^P mod P^2 (S words), c = CRT(c_p, c_q)
+template <int HS, int S>
+int run_encrypt_kh_dag(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                       uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  Scratch s_r, s_y, s_out;
+  int rc = s_y.alloc((size_t)2 * count * HS * 4, st);
+  if (rc) return rc;
+  rc = s_out.alloc((size_t)2 * count * S * 4, st);
+  if (rc) return rc;
+  flb::tc::ExpArgs A1, A2;
+  rc = tc_stage1_args<HS>(V, dev, r, seed, ctr0, (uint32_t*)s_y.p, count, st, s_r, A1);
+  if (rc) return rc;
+  tc_stage2_args<S>(V, dev, m, (const uint32_t*)s_y.p, (uint32_t*)s_out.p, count, A2);
+  rc = launch_tc_exp_dag<HS, S>(A1, A2, st);
+  if (rc) return rc;
+  return tc_combine<S>(V, dev, (const uint32_t*)s_out.p, c, count, st);
 }
 
 // decryption with both exponentiations c^(P-1) mod P^2 on the tensor cores (one launch), then the
@@ -869,6 +976,10 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
                                              size_t, cudaStream_t);                                              \
   EXT template int flb_rt::run_tc_debug_product<S>(const uint32_t*, const uint32_t*, uint32_t*, uint32_t, int,   \
                                                    cudaStream_t);
+#define FLB_TC_DAG_DECLS(EXT)                                                                                      \
+  EXT template int flb_rt::run_encrypt_kh_dag<32, 64>(const flb_priv*, const uint32_t*, const uint32_t*,         \
+                                                      const uint32_t*, uint64_t, uint64_t, uint32_t*, size_t,     \
+                                                      cudaStream_t);
 
 #ifndef FLB_INST_TU
 #define FLB_EXTERN_ENC(X, T) FLB_ENC_DECLS(extern, X, T)
@@ -877,6 +988,7 @@ FLB_ENC_COMBOS(FLB_EXTERN_ENC)
 FLB_DEC_COMBOS(FLB_EXTERN_DEC)
 FLB_TC_DECLS(extern, 32)
 FLB_TC_DECLS(extern, 64)
+FLB_TC_DAG_DECLS(extern)
 #undef FLB_EXTERN_ENC
 #undef FLB_EXTERN_DEC
 #endif

@@ -13,6 +13,9 @@ FLB_DEC_DECLS(, FLB_INST_X, FLB_INST_T)
 #endif
 #if defined(FLB_INST_TC)
 FLB_TC_DECLS(, FLB_INST_TC)
+#if FLB_INST_TC == 64
+FLB_TC_DAG_DECLS()
+#endif
 #endif
 
 #if defined(FLB_INST_TC) && FLB_INST_TC == 64 && FLB_TC_PROF

@@ -904,34 +904,106 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
   fence_async_smem();
 }
 
+// One tile (128 elements) of problem P: the element powers x^E (or (1 + m n) x^E) into P.out.  `tab`
+// is the CTA's window-table scratch ([entry][kTileM][S] words).  The Toeplitz operands of P are in
+// shared memory (tc_load_operands).
+template <int S>
+__device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, const uint32_t* one, uint32_t* tab,
+                                            const Smem& sm, uint32_t& phase) {
+  const Src row = src_row();
+  const int TB = P.table;
+  auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
+  auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
+  const uint64_t e0 = tile * kTileM;
+  const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
+  const uint32_t* xb = P.x + e0 * P.x_stride;
+  if (P.x_words <= (uint32_t)S) {
+    tc_mont<S>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+  } else {
+    tc_mont<S>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
+    tc_mont<S>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
+               phase);                                      // hi R^2
+    tc_row_add<S>(sm, slot(0), P.N);
+  }
+  tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
+  if (TB > 1) {
+    tc_mont<S>(row, row, true, sm, P.N, phase);             // x^2
+    tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
+#pragma unroll 1
+    for (int t = 1; t < TB; t++) {
+      tc_mont<S>(slot(t - 1), slot(TB), false, sm, P.N, phase);
+      tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
+    }
+  }
+  const uint32_t op0 = __ldg(P.sched);
+  Src cur = slot((int)(op0 >> 16) - 1);
+#pragma unroll 1
+  for (int o = 1; o < P.sched_len; o++) {
+    const uint32_t op = __ldg(P.sched + o);
+    const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
+#pragma unroll 1
+    for (int t = 0; t < sq; t++) {
+      tc_mont<S>(cur, cur, true, sm, P.N, phase);
+      cur = row;
+    }
+    if (idx >= 0) {
+      tc_mont<S>(cur, slot(idx), false, sm, P.N, phase);
+      cur = row;
+    }
+  }
+  if (P.m) {
+    tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
+    tc_mont<S>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
+    tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
+    tc_mont<S>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
+  } else {
+    tc_mont<S>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
+  }
+  tc_row_store<S>(sm, P.out + e0 * S, S, nvalid);
+}
+
+// CTA prologue / epilogue shared by the modexp kernels: the MMA-completion mbarrier and COLS TMEM columns
+template <int COLS>
+__device__ __forceinline__ void tc_cta_init(uint64_t* mbar, uint32_t* tmem_sh) {
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(mbar)));
+    asm volatile("fence.mbarrier_init.release.cluster;");
+  }
+  if ((threadIdx.x >> 5) == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" :: "r"(smem_u32(tmem_sh)),
+                 "n"(COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_before_sync();
+  __syncthreads();
+  tc_after_sync();
+}
+template <int COLS>
+__device__ __forceinline__ void tc_cta_fini(uint32_t tmem) {
+  tc_before_sync();
+  __syncthreads();
+  if ((threadIdx.x >> 5) == 0) {
+    tc_after_sync();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "n"(COLS));
+  }
+}
+
 template <int S>
 __global__ void __launch_bounds__(kThreads, 2) k_tc_exp(const ExpArgs A) {
   using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t tmem_sh;
-  const int tid = threadIdx.x, warp = tid >> 5;
-  if (tid == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(smem_u32(&mbar)));
-    asm volatile("fence.mbarrier_init.release.cluster;");
-  }
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" :: "r"(smem_u32(&tmem_sh)),
-                 "n"(C::TMEM_COLS));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  tc_before_sync();
-  __syncthreads();
-  tc_after_sync();
+  tc_cta_init<C::TMEM_COLS>(&mbar, &tmem_sh);
   const Smem sm{smem, tmem_sh, &mbar};
   uint32_t phase = 0;
   const uint64_t tiles_all = A.pb[0].tiles + (A.nprob > 1 ? A.pb[1].tiles : 0);
   int loaded = -1;
-  const Src row = src_row();
+  uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * A.tab_entries * S;
   for (uint64_t gt = blockIdx.x; gt < tiles_all; gt += gridDim.x) {
     const int pi = gt < A.pb[0].tiles ? 0 : 1;
     const ExpProblem& P = A.pb[pi];
-    const uint64_t tile = pi == 0 ? gt : gt - A.pb[0].tiles;
     if (pi != loaded) {
       __syncthreads();  // the previous problem's MMAs completed (waited on) before the overwrite
       tc_load_operands<S>(smem, P);
@@ -939,65 +1011,77 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp(const ExpArgs A) {
       __syncthreads();
       loaded = pi;
     }
-    const int TB = P.table;
-    uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * A.tab_entries * S;
-    auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
-    auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
-    const uint64_t e0 = tile * kTileM;
-    const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
-    const uint32_t* xb = P.x + e0 * P.x_stride;
-    if (P.x_words <= (uint32_t)S) {
-      tc_mont<S>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
-    } else {
-      tc_mont<S>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
-      tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
-      tc_mont<S>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
-                 phase);                                      // hi R^2
-      tc_row_add<S>(sm, slot(0), P.N);
-    }
-    tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
-    if (TB > 1) {
-      tc_mont<S>(row, row, true, sm, P.N, phase);             // x^2
-      tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
-#pragma unroll 1
-      for (int t = 1; t < TB; t++) {
-        tc_mont<S>(slot(t - 1), slot(TB), false, sm, P.N, phase);
-        tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
-      }
-    }
-    const uint32_t op0 = __ldg(P.sched);
-    Src cur = slot((int)(op0 >> 16) - 1);
-#pragma unroll 1
-    for (int o = 1; o < P.sched_len; o++) {
-      const uint32_t op = __ldg(P.sched + o);
-      const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
-#pragma unroll 1
-      for (int t = 0; t < sq; t++) {
-        tc_mont<S>(cur, cur, true, sm, P.N, phase);
-        cur = row;
-      }
-      if (idx >= 0) {
-        tc_mont<S>(cur, slot(idx), false, sm, P.N, phase);
-        cur = row;
-      }
-    }
-    if (P.m) {
-      tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
-      tc_mont<S>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
-      tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
-      tc_mont<S>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
-    } else {
-      tc_mont<S>(row, src_arr(A.one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
-    }
-    tc_row_store<S>(sm, P.out + e0 * S, S, nvalid);
+    tc_exp_tile<S>(P, pi == 0 ? gt : gt - A.pb[0].tiles, A.one, tab, sm, phase);
     __syncthreads();  // the work rows are rewritten by the next tile's first product
   }
-  tc_before_sync();
+  tc_cta_fini<C::TMEM_COLS>(tmem_sh);
+}
+
+// Key-holder encryption, both stages in one persistent launch (a dependency DAG instead of two
+// launches): the work queue holds the stage-1 tiles of A1 (y = r^Q mod P in the S1-word frame, both
+// primes) and then the stage-2 tiles of A2 ((1 + m n) y^P mod P^2 in the S2-word frame), taken
+// dynamically from a global counter.  Stage-2 tile j reads exactly the rows stage-1 tile j wrote
+// (same counts, same tile numbering), so it waits for tile j's flag (release / acquire at gpu
+// scope).  Every stage-1 tile is dequeued before any stage-2 tile, by a running CTA, so the wait
+// always ends.  Compared with two launches, the last partial round of stage 1 no longer idles the
+// GPU and the end-of-launch tail is at most one stage-2 tile per CTA slot.
+// sync: [0] the tile counter, [1 + j] the flag of stage-1 tile j (zeroed before the launch).
+template <int S1, int S2>
+__global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, const ExpArgs A2, uint32_t* sync,
+                                                           uint64_t tab_stride) {
+  constexpr int COLS = Cfg<S1>::TMEM_COLS > Cfg<S2>::TMEM_COLS ? Cfg<S1>::TMEM_COLS : Cfg<S2>::TMEM_COLS;
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ __align__(8) uint64_t mbar;
+  __shared__ uint32_t tmem_sh, next;
+  tc_cta_init<COLS>(&mbar, &tmem_sh);
+  const Smem sm{smem, tmem_sh, &mbar};
+  uint32_t phase = 0;
+  const uint64_t T1 = A1.pb[0].tiles + A1.pb[1].tiles, T2 = A2.pb[0].tiles + A2.pb[1].tiles;
+  int loaded = -1;  // 2 * stage + prime
+  uint32_t* tab = A1.scratch + (size_t)blockIdx.x * tab_stride;
+  if (threadIdx.x == 0) next = atomicAdd(sync, 1u);
   __syncthreads();
-  if (warp == 0) {
-    tc_after_sync();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem_sh), "n"(C::TMEM_COLS));
+  for (;;) {
+    const uint64_t gt = next;
+    if (gt >= T1 + T2) break;
+    const bool st2 = gt >= T1;
+    const uint64_t j = st2 ? gt - T1 : gt;
+    const ExpArgs& A = st2 ? A2 : A1;
+    const int pi = j < A.pb[0].tiles ? 0 : 1;
+    const ExpProblem& P = A.pb[pi];
+    const uint64_t tile = pi == 0 ? j : j - A.pb[0].tiles;
+    if (2 * (int)st2 + pi != loaded) {
+      __syncthreads();
+      if (st2) tc_load_operands<S2>(smem, P); else tc_load_operands<S1>(smem, P);
+      tc_before_sync();
+      __syncthreads();
+      loaded = 2 * (int)st2 + pi;
+    }
+    if (st2) {
+      if (threadIdx.x == 0) {
+        uint32_t f;
+        for (;;) {
+          asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(f) : "l"(sync + 1 + j) : "memory");
+          if (f) break;
+          __nanosleep(256);
+        }
+      }
+      __syncthreads();
+      tc_exp_tile<S2>(P, tile, A2.one, tab, sm, phase);
+    } else {
+      tc_exp_tile<S1>(P, tile, A1.one, tab, sm, phase);
+    }
+    __syncthreads();  // the tile's output rows are stored; the work rows are rewritten next
+    if (threadIdx.x == 0) {
+      if (!st2) {
+        __threadfence();
+        asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(sync + 1 + j), "r"(1u) : "memory");
+      }
+      next = atomicAdd(sync, 1u);
+    }
+    __syncthreads();
   }
+  tc_cta_fini<COLS>(tmem_sh);
 }
 
 // debug: the product phase alone (t = a b, or a^2 when sq) for up to 128 elements -> t [count][2S]

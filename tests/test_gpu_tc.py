@@ -190,3 +190,42 @@ def test_tc_product_phase_exact(words, square):
     for i in range(count):
         want = rnd[i] * (rnd[i] if square else other[i])
         assert t[i] == want, (i, hex(t[i] ^ want))
+
+
+def _env_run(fn, env):
+    old = {k: os.environ.get(k) for k in env}
+    try:
+        os.environ.update(env)
+        out = fn()
+        torch.cuda.synchronize()
+        return out
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+
+
+@pytest.mark.parametrize("count", [1, 129, 300, 20000])
+def test_tc_dag_launch_matches_two_launches_and_oracle(k2048, count):
+    """Both key-holder stages in one k_tc_exp_dag launch (dynamic tile queue, stage-2 tiles wait on
+    their stage-1 tile's flag): same ciphertexts as the two k_tc_exp launches (FLB_TC_DAG=0), as the
+    CIOS kernels, and as the oracle's Eq. 3 on sampled elements.  count = 20000 gives several tiles
+    of both stages per CTA (4 x 157 tiles on 296 CTAs), so stage-2 tiles run on other CTAs than the
+    stage-1 tiles they read."""
+    pub, priv, p, q = k2048
+    n = p * q
+    m_int = synthetic.uniform_below(n, min(count, 64), 900 + count)
+    m_int = (m_int * ((count + len(m_int) - 1) // len(m_int)))[:count]
+    m = to_dev(m_int, pub.pt_words)
+    seed, ctr0 = 0x5DA60000 + count, 3
+    dag = _env_run(lambda: flb.encrypt_crt(priv, m, seed=seed, ctr0=ctr0), {"FLB_TC": "1", "FLB_TC_DAG": "1"})
+    two = _env_run(lambda: flb.encrypt_crt(priv, m, seed=seed, ctr0=ctr0), {"FLB_TC": "1", "FLB_TC_DAG": "0"})
+    assert torch.equal(dag, two)
+    if count <= 300:
+        cios = _env_run(lambda: flb.encrypt_crt(priv, m, seed=seed, ctr0=ctr0), {"FLB_TC": "0"})
+        assert torch.equal(dag, cios)
+    got = from_dev(dag)
+    for i in sorted({0, count // 3, count - 1}):
+        assert got[i] == paillier.encrypt(n, m_int[i], philox.draw_r(n, seed, ctr0 + i, pub.pt_words)), i
