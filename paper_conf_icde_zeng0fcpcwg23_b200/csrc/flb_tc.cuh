@@ -196,6 +196,9 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
 #ifndef FLB_TC_SQR
 #define FLB_TC_SQR 1  // block squaring in the product phase (0: squarings use the general product)
 #endif
+#ifndef FLB_TC_CHAIN
+#define FLB_TC_CHAIN 1  // carry chains of the squaring's in-place additions as add.cc/addc.cc (0: 64-bit sums)
+#endif
 #ifndef FLB_TC_SQR32
 #define FLB_TC_SQR32 1  // block squaring also at S = 32 (two lanes per element)
 #endif
@@ -238,9 +241,33 @@ __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, i
                : reinterpret_cast<uint4*>(sW + elem * C::WROW + (w - S));
 }
 
-// t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2)
+// t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2).  One carry
+// chain (add.cc / addc.cc, one IADD3.X per word) across the chunks; the doubling is a funnel shift.
 template <int S, int NW>
 __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int elem, int w0, const uint32_t (&v)[NW]) {
+#if FLB_TC_CHAIN
+  uint32_t prev = 0, cy;
+#pragma unroll
+  for (int c = 0; c < NW / 4; c++) {
+    uint4* p = t_chunk<S>(sA, sW, elem, w0 + 4 * c);
+    const uint4 m = *p;
+    const uint32_t mm[4] = {m.x, m.y, m.z, m.w};
+    uint32_t r[4];
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t x = v[4 * c + u];
+      const uint32_t d = __funnelshift_l(prev, x, 1);  // (x << 1) | (prev >> 31)
+      prev = x;
+      if (c == 0 && u == 0)
+        asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(r[u]) : "r"(mm[u]), "r"(d));
+      else
+        asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(r[u]) : "r"(mm[u]), "r"(d));
+    }
+    *p = make_uint4(r[0], r[1], r[2], r[3]);
+  }
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
+  return cy + (prev >> 31);
+#else
   uint64_t cy = 0;
   uint32_t prev = 0;
 #pragma unroll
@@ -261,6 +288,34 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
     *p = make_uint4(r[0], r[1], r[2], r[3]);
   }
   return (uint32_t)cy + (prev >> 31);
+#endif
+}
+
+// q[j0 .. N) += the small addends add(j) (each < 2^32, nonzero at a few positions) with one carry
+// chain; returns the carry out of q[N - 1]
+template <int N, int J0, typename F>
+__device__ __forceinline__ uint32_t add_sparse_chain(uint32_t (&q)[N], F add) {
+#if FLB_TC_CHAIN
+  uint32_t cy;
+#pragma unroll
+  for (int j = J0; j < N; j++) {
+    if (j == J0)
+      asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(q[j]) : "r"(add(j)));
+    else
+      asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(q[j]) : "r"(add(j)));
+  }
+  asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
+  return cy;
+#else
+  uint64_t cy = 0;
+#pragma unroll
+  for (int j = J0; j < N; j++) {
+    const uint64_t s = (uint64_t)q[j] + add(j) + cy;
+    q[j] = (uint32_t)s;
+    cy = s >> 32;
+  }
+  return (uint32_t)cy;
+#endif
 }
 
 template <int S>
@@ -320,14 +375,7 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
     const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c);
     q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
   }
-  uint64_t cy = 0;
-#pragma unroll
-  for (int j = 0; j < 2 * X; j++) {
-    const uint32_t add = j == 0 ? at0 : j == X ? atX : j == X + H ? atH : 0u;
-    const uint64_t s = (uint64_t)q[j] + add + cy;
-    q[j] = (uint32_t)s;
-    cy = s >> 32;
-  }
+  const uint32_t cy = add_sparse_chain<2 * X, 0>(q, [&](int j) { return j == 0 ? at0 : j == X ? atX : j == X + H ? atH : 0u; });
   const uint32_t c = group_carry<kT>(cy != 0, all_ones<2 * X>(q), 0);
   add_word_propagate<2 * X>(q, c & 1u);
 #pragma unroll
@@ -374,13 +422,7 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
       const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X + 4 * c);
       q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
     }
-    uint64_t cy = 0;
-#pragma unroll
-    for (int j = H; j < 2 * X; j++) {
-      const uint64_t s = (uint64_t)q[j] + (j == H ? c0 : 0u) + (j == X ? cx : 0u) + cy;
-      q[j] = (uint32_t)s;
-      cy = s >> 32;
-    }
+    add_sparse_chain<2 * X, H>(q, [&](int j) { return j == H ? c0 : j == X ? cx : 0u; });  // (no carry leaves t)
 #pragma unroll
     for (int c = H / 4; c < X / 2; c++)
       *t_chunk<S>(sA, sW, elem, 2 * X + 4 * c) = make_uint4(q[4 * c], q[4 * c + 1], q[4 * c + 2], q[4 * c + 3]);
