@@ -140,6 +140,60 @@ __device__ __forceinline__ uint64_t word_of(uint32_t c0, uint32_t c1, uint32_t c
   return (uint64_t)c0 + ((uint64_t)c1 << 8) + ((uint64_t)c2 << 16) + ((uint64_t)c3 << 24);
 }
 
+// carry-flag chains (one IADD3(.X) per word; the flag lives between consecutive asm statements,
+// which no other instruction of this file touches)
+__device__ __forceinline__ uint32_t add_cc(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint32_t addc_cc(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint32_t addc_end(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("addc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint32_t sub_cc(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("sub.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint32_t subc_cc(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("subc.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__device__ __forceinline__ uint32_t subc_end(uint32_t a, uint32_t b) {
+  uint32_t r;
+  asm volatile("subc.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+
+// Normalise 8 words of byte-column sums (plus optional addends th) into v[0..8): with the 64-bit
+// word values W_w = word_of(cols 4w..4w+3) (+ th[w]), off the chain, the sum is
+// sum_w (lo W_w + hi W_(w-1)) 2^(32w), one addc.cc per word; `hprev` carries hi W of the last word
+// into the next chunk (the flag carries the rest).  first: the chain starts here (add.cc).
+template <bool TH>
+__device__ __forceinline__ void norm8_chain(const uint32_t (&cv)[32], const uint32_t* th, uint32_t* v,
+                                            uint32_t& hprev, bool first) {
+  uint32_t lo[8], hi[8];
+#pragma unroll
+  for (int w = 0; w < 8; w++) {
+    uint64_t W = word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]);
+    if (TH) W += th[w];
+    lo[w] = (uint32_t)W;
+    hi[w] = (uint32_t)(W >> 32);
+  }
+  v[0] = first ? add_cc(lo[0], hprev) : addc_cc(lo[0], hprev);
+#pragma unroll
+  for (int w = 1; w < 8; w++) v[w] = addc_cc(lo[w], hi[w - 1]);
+  hprev = hi[7];
+}
+
 struct Smem {
   uint8_t* base;
   uint32_t tmem;
@@ -668,12 +722,19 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   TC_MARK(1);
   uint32_t v[QW];
   auto add_in = [&](uint64_t cin) {
+#if FLB_TC_CHAIN
+    v[0] = add_cc(v[0], (uint32_t)cin);
+    v[1] = addc_cc(v[1], (uint32_t)(cin >> 32));
+#pragma unroll
+    for (int w = 2; w < QW; w++) v[w] = addc_cc(v[w], 0u);
+#else
 #pragma unroll
     for (int w = 0; w < QW; w++) {
       const uint64_t s = (uint64_t)v[w] + cin;
       v[w] = (uint32_t)s;
       cin = s >> 32;
     }
+#endif
   };
   auto publish = [&](uint64_t carry) {
     uint32_t ao = 0xffffffffu;
@@ -689,6 +750,17 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   };
   // ---- N1: q = D1 mod R
   {
+#if FLB_TC_CHAIN
+    uint32_t hprev = 0;
+#pragma unroll
+    for (int c0 = 0; c0 < QC; c0 += 32) {
+      uint32_t cv[32];
+      tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
+      tmem_wait();
+      norm8_chain<false>(cv, nullptr, v + c0 / 4, hprev, c0 == 0);
+    }
+    publish(addc_end(hprev, 0u));
+#else
     uint64_t carry = 0;
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
@@ -703,6 +775,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       }
     }
     publish(carry);
+#endif
   }
   tc_before_sync();
   __syncthreads();  // D1 drained, t_lo bytes read, carries published
@@ -737,6 +810,9 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       const uint64_t s1 = (s0 >> 32) + word_of(bc[4], bc[5], bc[6], bc[7]) + ttop.y;
       carry = (s1 >> 32) + ((((uint32_t)s0) | ((uint32_t)s1)) != 0u ? 1u : 0u);
     }
+#if FLB_TC_CHAIN
+    uint32_t hprev = (uint32_t)carry;  // < 2^20
+#endif
     // this half's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; half 1's last 8 columns
     // (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
     uint32_t top[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -778,14 +854,22 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       const uint4 h0 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[0];
       const uint4 h1 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[1];
       const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
+#if FLB_TC_CHAIN
+      norm8_chain<true>(cv, th, v + c0 / 4, hprev, c0 == 0);
+#else
 #pragma unroll
       for (int w = 0; w < 8; w++) {
         const uint64_t s = carry + word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]) + th[w];
         v[c0 / 4 + w] = (uint32_t)s;
         carry = s >> 32;
       }
+#endif
     }
+#if FLB_TC_CHAIN
+    publish(addc_end(hprev, 0u));
+#else
     publish(carry);
+#endif
   }
   tc_before_sync();
   __syncthreads();
@@ -796,6 +880,20 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   uint32_t d[QW];
   {
     uint32_t br = 0, nzd = 0;
+#if FLB_TC_CHAIN
+    uint32_t nn[QW];
+#pragma unroll
+    for (int c = 0; c < QW / 4; c++) {
+      const uint4 nv = __ldg(reinterpret_cast<const uint4*>(Nmod + g * QW + 4 * c));
+      nn[4 * c] = nv.x; nn[4 * c + 1] = nv.y; nn[4 * c + 2] = nv.z; nn[4 * c + 3] = nv.w;
+    }
+    d[0] = sub_cc(v[0], nn[0]);
+#pragma unroll
+    for (int w = 1; w < QW; w++) d[w] = subc_cc(v[w], nn[w]);
+    br = subc_end(0u, 0u) & 1u;
+#pragma unroll
+    for (int w = 0; w < QW; w++) nzd |= d[w];
+#else
 #pragma unroll
     for (int c = 0; c < QW / 4; c++) {
       const uint4 nv = __ldg(reinterpret_cast<const uint4*>(Nmod + g * QW + 4 * c));
@@ -808,6 +906,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
         nzd |= (uint32_t)df;
       }
     }
+#endif
     xch[g].w = br | (nzd == 0u ? 2u : 0u);
   }
   __syncthreads();
@@ -816,6 +915,11 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     const uint32_t b1 = f0 & 1u;                          // borrow into half 1
     const uint32_t bout = (f1 & 1u) | ((f1 >> 1) & b1);    // borrow out of the top
     if (ovf != 0 || bout == 0) {                           // u >= N: take u - N
+#if FLB_TC_CHAIN
+      v[0] = sub_cc(d[0], g == 1 ? b1 : 0u);
+#pragma unroll
+      for (int w = 1; w < QW; w++) v[w] = subc_cc(d[w], 0u);
+#else
       uint32_t br = g == 1 ? b1 : 0u;
 #pragma unroll
       for (int w = 0; w < QW; w++) {
@@ -823,6 +927,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
         v[w] = (uint32_t)df;
         br = (uint32_t)(df >> 63);
       }
+#endif
     }
 #pragma unroll
     for (int c = 0; c < QW / 4; c++)
