@@ -255,6 +255,17 @@ static uint64_t tc_imad_lp(uint64_t S, uint64_t mults, uint64_t sqr) {
   return (mults - sqr) * S * S + sqr * sq_lp;
 }
 
+// u8 MACs the two Toeplitz MMAs of one S-word tensor-core Montgomery product issue per element (MMA
+// row): K-slices of 32 bytes, q = t N' mod R over columns [32 ks, KB), q N over [0, min(KB, 32 ks + 48))
+// (flb_tc.cuh mma_toeplitz_lo / _hi; 2 KB^2 with FLB_TC_TRI=0)
+static uint64_t tc_mma_macs(uint64_t S) {
+  const uint64_t KB = 4 * S;
+  if (!FLB_TC_TRI) return 2 * KB * KB;
+  uint64_t m = 0;
+  for (uint64_t ks = 0; ks < KB / 32; ks++) m += 32 * (KB - 32 * ks) + 32 * std::min<uint64_t>(KB, 32 * ks + 48);
+  return m;
+}
+
 int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls, uint64_t* limb_products) {
   if (!mont_muls || !limb_products) return fail(FLB_EINVAL, "null output");
   const flb_pub* P = K ? K : (V ? V->pub : nullptr);
@@ -319,7 +330,8 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       *limb_products = tc_imad_lp(sp, mm, sq);
       return FLB_OK;
     }
-    case 7:    // key-holder encryption, tensor-core kernels: *limb_products = u8 MACs (2 KB^2 per product)
+    case 7:    // key-holder encryption, tensor-core kernels: *limb_products = u8 MACs the MMAs issue per element
+               // (triangular K-slices, tc_mma_macs)
     case 8: {  // decryption exponentiations, tensor-core kernel: likewise
       uint64_t mm, lp;
       const int rc = flb_op_cost(K, V, op - 2, &mm, &lp);
@@ -327,9 +339,9 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       if (op == 7) {
         const uint64_t h = V->H;
         const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
-        *limb_products = 32 * (s1 * h * h + (mm - s1) * sp * sp);
+        *limb_products = s1 * tc_mma_macs(h) + (mm - s1) * tc_mma_macs(sp);
       } else {
-        *limb_products = 32 * mm * sp * sp;
+        *limb_products = mm * tc_mma_macs(sp);
       }
       *mont_muls = mm;
       return FLB_OK;

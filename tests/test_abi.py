@@ -186,8 +186,7 @@ def _sliding_counts(e, w):
 def test_op_cost_tensor_core_paths():
     """Accounting of the tensor-core kernels (bench.py's roofline): Montgomery products per element,
     IMAD-pipe limb products (S^2 per product; block squaring 10 (S/4)^2 at S = 64, 3 (S/2)^2 at
-    S = 32) and u8 MACs
-    (2 (4S)^2 per product), against an independent window count."""
+    S = 32) and the u8 MACs the triangular Toeplitz MMAs issue, against an independent window count."""
     p, q = KEYS["2048"]
     pub, priv = flb.key_from_primes(p, q)
     sp, h = 64, 32
@@ -201,7 +200,16 @@ def test_op_cost_tensor_core_paths():
     (mp, sqp), (mq, sqq) = best(p - 1), best(q - 1)
     assert mm == mp + mq + 2 * 3
     assert any(lp == (mm - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in sqp for b in sqq)
-    assert flb.op_cost(priv, "decrypt_tc_macs") == (mm, 32 * mm * sp * sp)
+    def macs(S):
+        # (K, column) pairs the triangular K-slices cover: q = t N' mod R reaches column j from
+        # K <= j; the high half of q N (columns KB-8+j) from K >= j - 39 within the slice's 32 rows
+        KB = 4 * S
+        lo = sum(32 * (KB - 32 * ks) for ks in range(KB // 32))
+        hi = sum(32 * min(KB, 32 * ks + 48) for ks in range(KB // 32))
+        assert lo < KB * KB and hi < KB * KB
+        return lo + hi
+
+    assert flb.op_cost(priv, "decrypt_tc_macs") == (mm, mm * macs(sp))
     mm_e, lp_e = flb.op_cost(priv, "encrypt_crt_tc")
     (ep, esp), (eq, esq) = best(p), best(q)
     s1 = (2 + eq + 1) + (2 + ep + 1)      # stage 1: r^Q mod p, r^P mod q at the half frame
@@ -210,7 +218,7 @@ def test_op_cost_tensor_core_paths():
     # stage 1 (h = 32 words, two lanes): squarings 3 (h/2)^2; stage 2 (64 words, four lanes): 10 (sp/4)^2
     assert any(lp_e == (s1 - a - b) * h * h + (a + b) * 3 * (h // 2) ** 2
                + (s2 - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in esp for b in esq)
-    assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, 32 * (s1 * h * h + s2 * sp * sp))
+    assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, s1 * macs(h) + s2 * macs(sp))
     # 1024-bit keys have no two-stage (half-frame) encryption path
     p1, q1 = KEYS["1024"]
     _, priv1 = flb.key_from_primes(p1, q1)
