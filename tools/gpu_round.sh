@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round-end style GPU session: parity suite, smoke, every bench config, the C2 launch list, and one
-# ncu --set full capture per tensor-core kernel of the C2 step (stage 1, stage 2, decryption; one
+# ncu --set full capture per tensor-core kernel of the C2 step (encryption, decryption; one
 # process each).  Outputs under gpurun_out/${TAG}_*.
 set -u
 TAG=${TAG:-round}
@@ -14,8 +14,10 @@ done
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e \
   > gpurun_out/${TAG}_bench_under_ncu.log 2>&1
+# prof_c2.py launches the key-holder encryption (k_tc_exp_dag: both stages, one launch) first, then
+# the decryption (k_tc_exp<64>); FLB_TC_DAG=0 gives the two-launch form (stage 1, stage 2, decryption)
 i=0
-for name in stage1 stage2 decrypt; do
+for name in encrypt decrypt; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_tc_exp --launch-skip $i -c 1 \
     -o gpurun_out/${TAG}_ncu_$name python tools/prof_c2.py > gpurun_out/${TAG}_ncu_$name.log 2>&1
   i=$((i + 1))
