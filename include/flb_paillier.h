@@ -275,7 +275,7 @@ int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint
  * u8 MMAs, PAPER Alg. 1 L98-L114 restated as a contraction against the shared modulus), whose IMAD
  * work is only the S^2 limb products of t = a b per S-word multiplication: 5 = key-holder encrypt
  * (both stages, priv), 6 = decrypt's two exponentiations (priv); *limb_products = those
- * products on the IMAD pipe (S^2 per product, 10 (S/4)^2 per block squaring at S >= 64);
+ * products on the IMAD pipe (S^2 per product, S (S + 1) / 2 per block squaring);
  * 7 / 8 = the same two ops with *limb_products = their u8 MMA MACs (2 (4S)^2 per product).
  * Host only.  Errors: FLB_EINVAL; FLB_EUNSUPPORTED for ops 5/6 on keys without the path. */
 int flb_op_cost(const flb_pub* pub, const flb_priv* priv, int op, uint64_t* mont_muls,

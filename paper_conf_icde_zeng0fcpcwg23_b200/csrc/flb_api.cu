@@ -246,12 +246,15 @@ static uint64_t sched_squarings(const H::Schedule& S) {
 }
 
 // IMAD-pipe limb products of the tensor-core kernel (flb_tc.cuh) for `mults` S-word Montgomery
-// products of which `sqr` are squarings: S^2 for the row-scan product, 10 (S/4)^2 for the block
-// squaring on 4 lanes (S >= 64), 3 (S/2)^2 on 2 lanes (S = 32)
+// products of which `sqr` are squarings: S^2 for the row-scan product; for the block squaring
+// (S >= 64 on 4 lanes, S = 32 on 2) S (S + 1) / 2 with triangular diagonal blocks (FLB_TC_TRISQ),
+// else 10 (S/4)^2 on 4 lanes, 3 (S/2)^2 on 2
 static uint64_t tc_imad_lp(uint64_t S, uint64_t mults, uint64_t sqr) {
-  const uint64_t sq_lp = (FLB_TC_SQR && S >= 64)    ? 10 * (S / 4) * (S / 4)
-                         : (FLB_TC_SQR && FLB_TC_SQR32) ? 3 * (S / 2) * (S / 2)
-                                                         : S * S;
+  const bool blk = FLB_TC_SQR && (S >= 64 || FLB_TC_SQR32);
+  const uint64_t sq_lp = !blk           ? S * S
+                         : FLB_TC_TRISQ ? S * (S + 1) / 2
+                         : S >= 64      ? 10 * (S / 4) * (S / 4)
+                                        : 3 * (S / 2) * (S / 2);
   return (mults - sqr) * S * S + sqr * sq_lp;
 }
 

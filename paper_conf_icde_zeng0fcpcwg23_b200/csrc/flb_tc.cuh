@@ -321,6 +321,58 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
   for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(out[R + t]) : "r"(E[t]), "r"(O[t - 1]));
 }
 
+#ifndef FLB_TC_TRISQ
+#define FLB_TC_TRISQ 1  // diagonal blocks a_k^2 as lane-local triangular squares (0: full X x X blk_prod)
+#endif
+
+// v = a^2 (2X words) for this lane's own block, X (X - 1) / 2 + X limb products instead of X^2
+// (squarings dominate the modexp).  U = sum_{i<j} a_i a_j 2^(32 (i + j)) by rows
+// j = 0 .. X - 2 (row j: a[j+1, X) x a_j at word 2j + 1, a lo chain then a hi chain one word up),
+// then v = 2 U + sum_i a_i^2 2^(64 i) in one carry chain with the doubling as a funnel shift.
+// Bounds: after row j the partial sum is < 2^(32 (X + j + 1)), so neither chain carries past word
+// X + j + 1; 2 U + D = a^2 < 2^(64 X), so the final chain has no carry out.
+template <int X>
+__device__ __forceinline__ void sqr_local(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
+  uint32_t u[2 * X];
+#pragma unroll
+  for (int w = 0; w < 2 * X; w++) u[w] = 0;
+#pragma unroll
+  for (int j = 0; j < X - 1; j++) {
+    // lo chain: u[i + j] += lo(a_i a_j), i = j+1 .. X-1; carry into u[X + j] (<= 1 before: no carry out)
+#pragma unroll
+    for (int i = j + 1; i < X; i++) {
+      if (i == j + 1)
+        asm volatile("mad.lo.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j]) : "r"(a[i]), "r"(a[j]));
+      else
+        asm volatile("madc.lo.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j]) : "r"(a[i]), "r"(a[j]));
+    }
+    asm volatile("addc.u32 %0, %0, 0;" : "+r"(u[X + j]));
+    // hi chain: u[i + j + 1] += hi(a_i a_j); carry into the fresh word u[X + j + 1]
+#pragma unroll
+    for (int i = j + 1; i < X; i++) {
+      if (i == j + 1)
+        asm volatile("mad.hi.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j + 1]) : "r"(a[i]), "r"(a[j]));
+      else
+        asm volatile("madc.hi.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j + 1]) : "r"(a[i]), "r"(a[j]));
+    }
+    asm volatile("addc.u32 %0, 0, 0;" : "=r"(u[X + j + 1]));
+  }
+  // v = 2 U + D
+#pragma unroll
+  for (int i = 0; i < X; i++) {
+    const uint32_t d0 = __funnelshift_l(i == 0 ? 0u : u[2 * i - 1], u[2 * i], 1);
+    const uint32_t d1 = __funnelshift_l(u[2 * i], u[2 * i + 1], 1);
+    if (i == 0)
+      asm volatile("mad.lo.cc.u32 %0, %1, %1, %2;" : "=r"(v[0]) : "r"(a[0]), "r"(d0));
+    else
+      asm volatile("madc.lo.cc.u32 %0, %1, %1, %2;" : "=r"(v[2 * i]) : "r"(a[i]), "r"(d0));
+    if (i == X - 1)
+      asm volatile("madc.hi.u32 %0, %1, %1, %2;" : "=r"(v[2 * i + 1]) : "r"(a[i]), "r"(d1));
+    else
+      asm volatile("madc.hi.cc.u32 %0, %1, %1, %2;" : "=r"(v[2 * i + 1]) : "r"(a[i]), "r"(d1));
+  }
+}
+
 // address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work row
 template <int S>
 __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, int w) {
@@ -415,7 +467,7 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
   {
     // diagonal block: t[2Xk, 2Xk + 2X) = a_k^2 (the four tile t exactly)
     uint32_t v[2 * X];
-    blk_prod<X, X>(v, a, a, k, false);
+    if (FLB_TC_TRISQ) sqr_local<X>(v, a); else blk_prod<X, X>(v, a, a, k, false);
     __syncwarp();  // every lane of the group has read its a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -482,7 +534,7 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
   const int k = threadIdx.x % 2;
   {
     uint32_t v[2 * X];
-    blk_prod<X, X, 2>(v, a, a, k, false);
+    if (FLB_TC_TRISQ) sqr_local<X>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
     __syncwarp();  // both lanes have read a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)

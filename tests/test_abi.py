@@ -185,8 +185,9 @@ def _sliding_counts(e, w):
 
 def test_op_cost_tensor_core_paths():
     """Accounting of the tensor-core kernels (bench.py's roofline): Montgomery products per element,
-    IMAD-pipe limb products (S^2 per product; block squaring 10 (S/4)^2 at S = 64, 3 (S/2)^2 at
-    S = 32) and the u8 MACs the triangular Toeplitz MMAs issue, against an independent window count."""
+    IMAD-pipe limb products (S^2 per product; block squaring with triangular diagonal blocks:
+    4 x (X (X + 1) / 2 + 1.5 X^2) at S = 64 (X = 16 limbs per lane), 2 x (X (X + 1) / 2 + X^2 / 2)
+    at S = 32) and the u8 MACs the triangular Toeplitz MMAs issue, against an independent window count."""
     p, q = KEYS["2048"]
     pub, priv = flb.key_from_primes(p, q)
     sp, h = 64, 32
@@ -199,7 +200,10 @@ def test_op_cost_tensor_core_paths():
     mm, lp = flb.op_cost(priv, "decrypt_tc")
     (mp, sqp), (mq, sqq) = best(p - 1), best(q - 1)
     assert mm == mp + mq + 2 * 3
-    assert any(lp == (mm - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in sqp for b in sqq)
+    X = 16  # limbs per lane at both frames
+    sq64 = 4 * (X * (X + 1) // 2 + X * X + X * X // 2)   # diagonal, full and half off-diagonal blocks
+    sq32 = 2 * (X * (X + 1) // 2 + X * X // 2)           # diagonal, half cross block
+    assert any(lp == (mm - a - b) * sp * sp + (a + b) * sq64 for a in sqp for b in sqq)
     def macs(S):
         # (K, column) pairs the triangular K-slices cover: q = t N' mod R reaches column j from
         # K <= j; the high half of q N (columns KB-8+j) from K >= j - 39 within the slice's 32 rows
@@ -215,9 +219,9 @@ def test_op_cost_tensor_core_paths():
     s1 = (2 + eq + 1) + (2 + ep + 1)      # stage 1: r^Q mod p, r^P mod q at the half frame
     s2 = (1 + ep + 2) + (1 + eq + 2)      # stage 2: y^P mod P^2
     assert mm_e == s1 + s2
-    # stage 1 (h = 32 words, two lanes): squarings 3 (h/2)^2; stage 2 (64 words, four lanes): 10 (sp/4)^2
-    assert any(lp_e == (s1 - a - b) * h * h + (a + b) * 3 * (h // 2) ** 2
-               + (s2 - a - b) * sp * sp + (a + b) * 10 * (sp // 4) ** 2 for a in esp for b in esq)
+    # stage 1 (h = 32 words, two lanes), stage 2 (64 words, four lanes)
+    assert any(lp_e == (s1 - a - b) * h * h + (a + b) * sq32
+               + (s2 - a - b) * sp * sp + (a + b) * sq64 for a in esp for b in esq)
     assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, s1 * macs(h) + s2 * macs(sp))
     # 1024-bit keys have no two-stage (half-frame) encryption path
     p1, q1 = KEYS["1024"]
