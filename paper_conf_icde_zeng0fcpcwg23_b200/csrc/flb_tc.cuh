@@ -383,7 +383,7 @@ __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, i
 
 // t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2).  One carry
 // chain (add.cc / addc.cc, one IADD3.X per word) across the chunks; the doubling is a funnel shift.
-template <int S, int NW>
+template <int S, int NW, bool DBL = true>
 __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int elem, int w0, const uint32_t (&v)[NW]) {
 #if FLB_TC_CHAIN
   uint32_t prev = 0, cy;
@@ -396,7 +396,7 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
 #pragma unroll
     for (int u = 0; u < 4; u++) {
       const uint32_t x = v[4 * c + u];
-      const uint32_t d = __funnelshift_l(prev, x, 1);  // (x << 1) | (prev >> 31)
+      const uint32_t d = DBL ? __funnelshift_l(prev, x, 1) : x;  // (x << 1) | (prev >> 31)
       prev = x;
       if (c == 0 && u == 0)
         asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(r[u]) : "r"(mm[u]), "r"(d));
@@ -406,7 +406,7 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
     *p = make_uint4(r[0], r[1], r[2], r[3]);
   }
   asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
-  return cy + (prev >> 31);
+  return cy + (DBL ? prev >> 31 : 0u);
 #else
   uint64_t cy = 0;
   uint32_t prev = 0;
@@ -419,7 +419,7 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
 #pragma unroll
     for (int u = 0; u < 4; u++) {
       const uint32_t x = v[4 * c + u];
-      d[u] = (x << 1) | (prev >> 31);
+      d[u] = DBL ? (x << 1) | (prev >> 31) : x;
       prev = x;
       const uint64_t s = (uint64_t)mm[u] + d[u] + cy;
       r[u] = (uint32_t)s;
@@ -427,7 +427,7 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
     }
     *p = make_uint4(r[0], r[1], r[2], r[3]);
   }
-  return (uint32_t)cy + (prev >> 31);
+  return (uint32_t)cy + (DBL ? prev >> 31 : 0u);
 #endif
 }
 
@@ -693,6 +693,111 @@ __device__ __forceinline__ void tc_square_product_reg(const uint32_t (&a)[Cfg<S>
     *t_chunk<S>(sA, sW, elem, Q * k + 4 * c) = make_uint4(acc[4 * c], acc[4 * c + 1], acc[4 * c + 2], acc[4 * c + 3]);
 }
 
+#ifndef FLB_TC_GBLK
+#define FLB_TC_GBLK 0  // general products as lane-local X x X blocks: bit-exact but 2.7 % slower (spills)
+#endif
+
+// t = a b for a != b by lane-local X x X block products (the general products of a modexp: window
+// table, multiply steps, epilogue).  Lane k holds a_k, b_k (X words each); in round d it computes
+// a_k b_((k+d) mod T) (rows of b by shuffle, one per row) and adds it at words X (k + (k+d) mod T).
+// T = 4: round 0 fills the four quarters t[2Xk, 2Xk + 2X); rounds 1, 3 cover [X, 3X), [3X, 5X),
+// [5X, 7X) plus a second [3X, 5X) piece (two phases each); round 2 covers [2X, 4X) and [4X, 6X) twice
+// (two phases).  T = 2: round 0 fills the halves, round 1 adds a_0 b_1 and a_1 b_0 at [X, 3X) (two
+// phases).  Each piece's carry-out (0/1) lands at a fixed word; one fold pass per quarter adds them,
+// its carries resolved by a ballot carry-lookahead.  T X^2 limb products per lane, as the row scan.
+template <int S>
+__device__ __forceinline__ void tc_general_product(const uint32_t (&a)[Cfg<S>::X], const uint32_t (&b)[Cfg<S>::X],
+                                                   int elem, uint8_t* sA, uint32_t* sW) {
+  constexpr int X = Cfg<S>::X, T = Cfg<S>::T;
+  const int k = threadIdx.x % T;
+  {
+    uint32_t v[2 * X];
+    blk_prod<X, X, T>(v, a, b, k, false);
+    __syncwarp();  // every lane has its a, b (they may come from the work row)
+#pragma unroll
+    for (int c = 0; c < X / 2; c++)
+      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  }
+  if constexpr (T == 2) {
+    uint32_t v[2 * X];
+    blk_prod<X, X, T>(v, a, b, k ^ 1, false);
+    uint32_t cx = 0;
+    __syncwarp();
+    if (k == 0) cx = t_add_dbl<S, 2 * X, false>(sA, sW, elem, X, v);
+    __syncwarp();
+    if (k == 1) cx = t_add_dbl<S, 2 * X, false>(sA, sW, elem, X, v);
+    __syncwarp();
+    const uint32_t c0 = __shfl_sync(FULL, cx, 0, 2);
+    if (k == 1) {  // both carries at word 3X = lane 1's relative X; no carry leaves t
+      uint32_t q[X];
+#pragma unroll
+      for (int c = 0; c < X / 4; c++) {
+        const uint4 u = *t_chunk<S>(sA, sW, elem, 3 * X + 4 * c);
+        q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
+      }
+      add_sparse_chain<X, 0>(q, [&](int j) { return j == 0 ? c0 + cx : 0u; });
+#pragma unroll
+      for (int c = 0; c < X / 4; c++)
+        *t_chunk<S>(sA, sW, elem, 3 * X + 4 * c) = make_uint4(q[4 * c], q[4 * c + 1], q[4 * c + 2], q[4 * c + 3]);
+    }
+    __syncwarp();
+  } else {
+    static_assert(T == 4, "block product on 2 or 4 lanes");
+    uint32_t c1 = 0, c2 = 0, c3 = 0;
+    {  // round 1: a_k b_(k+1): lanes 0-2 at X (2k + 1), lane 3 at 3X; carries at X (2k + 3), lane 3 at 5X
+      uint32_t v[2 * X];
+      blk_prod<X, X, T>(v, a, b, (k + 1) & 3, false);
+      const int w0 = X * (k < 3 ? 2 * k + 1 : 3);
+      __syncwarp();
+      if (k < 3) c1 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+      __syncwarp();
+      if (k == 3) c1 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+    }
+    {  // round 3: a_k b_(k-1): lanes 1-3 at X (2k - 1), lane 0 at 3X; carries at X (2k + 1), lane 0 at 5X
+      uint32_t v[2 * X];
+      blk_prod<X, X, T>(v, a, b, (k + 3) & 3, false);
+      const int w0 = X * (k > 0 ? 2 * k - 1 : 3);
+      __syncwarp();
+      if (k > 0) c3 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+      __syncwarp();
+      if (k == 0) c3 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+    }
+    {  // round 2: a_k b_(k+2): lanes 0, 2 at 2X, lanes 1, 3 at 4X; carries at 4X, 6X
+      uint32_t v[2 * X];
+      blk_prod<X, X, T>(v, a, b, (k + 2) & 3, false);
+      const int w0 = X * (2 + 2 * (k & 1));
+      __syncwarp();
+      if (k < 2) c2 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+      __syncwarp();
+      if (k >= 2) c2 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
+      __syncwarp();
+    }
+    // carries into quarter k ([2Xk, 2Xk + 2X)), at relative 0 and X:
+    //   q1: X <- c1(0) + c3(1);  q2: 0 <- c2(0) + c2(2), X <- c1(1) + c1(3) + c3(2) + c3(0);
+    //   q3: 0 <- c2(1) + c2(3), X <- c1(2) + c3(3)
+    const uint32_t a0 = __shfl_sync(FULL, c1, 0, T), a1 = __shfl_sync(FULL, c1, 1, T);
+    const uint32_t a2 = __shfl_sync(FULL, c1, 2, T), a3 = __shfl_sync(FULL, c1, 3, T);
+    const uint32_t b0 = __shfl_sync(FULL, c3, 0, T), b1 = __shfl_sync(FULL, c3, 1, T);
+    const uint32_t b2 = __shfl_sync(FULL, c3, 2, T), b3 = __shfl_sync(FULL, c3, 3, T);
+    const uint32_t d0 = __shfl_sync(FULL, c2, 0, T), d1 = __shfl_sync(FULL, c2, 1, T);
+    const uint32_t d2 = __shfl_sync(FULL, c2, 2, T), d3 = __shfl_sync(FULL, c2, 3, T);
+    const uint32_t at0 = k == 2 ? d0 + d2 : k == 3 ? d1 + d3 : 0u;
+    const uint32_t atX = k == 1 ? a0 + b1 : k == 2 ? a1 + a3 + b2 + b0 : k == 3 ? a2 + b3 : 0u;
+    uint32_t q[2 * X];
+#pragma unroll
+    for (int c = 0; c < X / 2; c++) {
+      const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c);
+      q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
+    }
+    const uint32_t cy = add_sparse_chain<2 * X, 0>(q, [&](int j) { return j == 0 ? at0 : j == X ? atX : 0u; });
+    const uint32_t c = group_carry<T>(cy != 0, all_ones<2 * X>(q), 0);
+    add_word_propagate<2 * X>(q, c & 1u);
+#pragma unroll
+    for (int cc = 0; cc < X / 2; cc++)
+      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
+  }
+}
+
 // The product phase of tc_mont: t = a b (2S words) for the 128 elements of the tile, t_lo into the
 // elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of T lanes per element
 // (X = 16 limbs each), NP passes of EP elements.  CTA-collective (no trailing barrier).
@@ -732,6 +837,10 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
       for (int j = 0; j < X; j++) b[j] = a[j];
     } else {
       src_load<S>(b, sb, elem, sW);
+      if constexpr (FLB_TC_GBLK) {
+        tc_general_product<S>(a, b, elem, sA, sW);
+        continue;
+      }
     }
     // stage b in the element's sA row (natural byte order: word w at chunk w / 4)
     __syncwarp();
