@@ -192,6 +192,29 @@ def test_tc_product_phase_exact(words, square):
         assert t[i] == want, (i, hex(t[i] ^ want))
 
 
+@pytest.mark.parametrize("words", [32, 64])
+def test_tc_square_block_carries(words):
+    """Block squaring with triangular diagonal blocks (sqr_local: sum_{i<j} a_i a_j by lo/hi row
+    chains, doubled, plus a_i^2): operands whose 16-limb lane blocks are all-ones, zero, or
+    alternate 0xffffffff / 1 limbs, so every row chain, the doubling's shifted-out bits and the
+    quarter carries hit their extremes; exact 2w-limb a^2."""
+    X, nb = 16, words // 16
+    full = (1 << (32 * X)) - 1
+    alt = sum((0xFFFFFFFF if j % 2 == 0 else 1) << (32 * j) for j in range(X))
+    alt2 = sum((1 if j % 2 == 0 else 0xFFFFFFFF) << (32 * j) for j in range(X))
+    vals = []
+    for blk in (full, alt, alt2, full - 1, 1 << (32 * X - 1)):
+        for kb in range(nb):
+            vals.append(blk << (32 * X * kb))                                  # one block set
+        vals.append(sum(blk << (32 * X * kb) for kb in range(nb)))             # every block
+        vals.append(sum(blk << (32 * X * kb) for kb in range(0, nb, 2)))       # alternate blocks
+    vals += synthetic.uniform_below(1 << (32 * words), 128 - len(vals), 7150 + words)
+    a = to_dev(vals, words)
+    t = from_dev(flb.debug_tc_product(a, a, square=True))
+    for i, v in enumerate(vals):
+        assert t[i] == v * v, (i, hex(t[i] ^ (v * v)))
+
+
 def _env_run(fn, env):
     old = {k: os.environ.get(k) for k in env}
     try:
