@@ -373,6 +373,52 @@ __device__ __forceinline__ void sqr_local(uint32_t (&v)[2 * X], const uint32_t (
   }
 }
 
+// FLB_TC_TRISQ == 2: a^2 = L^2 + 2 L H 2^(32 X/2) + H^2 2^(32 X) with a = L + H 2^(32 X/2): the two
+// half-size triangular squares are independent chains written to disjoint halves of v, the L H
+// block (X/2 rows of local_row, two chains per row) is doubled into words [X/2, 3X/2) with the carry
+// rippled to the top; the same X (X + 1) / 2 limb products as sqr_local<X>, more independent chains
+template <int X>
+__device__ __forceinline__ void sqr_local_split(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
+  constexpr int H = X / 2;
+  uint32_t lo[H], hi[H], sl[X], sh[X], m[X];
+#pragma unroll
+  for (int j = 0; j < H; j++) { lo[j] = a[j]; hi[j] = a[H + j]; }
+  sqr_local<H>(sl, lo);
+  sqr_local<H>(sh, hi);
+  {
+    uint32_t E[H + 1], O[H + 1], pend = 0;
+#pragma unroll
+    for (int t = 0; t <= H; t++) { E[t] = 0; O[t] = 0; }
+#pragma unroll
+    for (int j = 0; j < H; j++) m[j] = local_row<H>(E, O, pend, lo, hi[j]);
+    asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(m[H]) : "r"(E[0]), "r"(pend));
+#pragma unroll
+    for (int t = 1; t < H; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(m[H + t]) : "r"(E[t]), "r"(O[t - 1]));
+  }
+#pragma unroll
+  for (int i = 0; i < X; i++) { v[i] = sl[i]; v[X + i] = sh[i]; }
+  uint32_t prev = 0;
+#pragma unroll
+  for (int t = 0; t < X; t++) {
+    const uint32_t d = __funnelshift_l(prev, m[t], 1);
+    prev = m[t];
+    if (t == 0)
+      asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(v[H]) : "r"(d));
+    else
+      asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(v[H + t]) : "r"(d));
+  }
+  const uint32_t top = prev >> 31;
+  asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(v[H + X]) : "r"(top));
+#pragma unroll
+  for (int w = H + X + 1; w < 2 * X - 1; w++) asm volatile("addc.cc.u32 %0, %0, 0;" : "+r"(v[w]));
+  asm volatile("addc.u32 %0, %0, 0;" : "+r"(v[2 * X - 1]));
+}
+
+template <int X>
+__device__ __forceinline__ void sqr_diag(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
+  if constexpr (FLB_TC_TRISQ == 2) sqr_local_split<X>(v, a); else sqr_local<X>(v, a);
+}
+
 // address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work row
 template <int S>
 __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, int w) {
@@ -467,7 +513,7 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
   {
     // diagonal block: t[2Xk, 2Xk + 2X) = a_k^2 (the four tile t exactly)
     uint32_t v[2 * X];
-    if (FLB_TC_TRISQ) sqr_local<X>(v, a); else blk_prod<X, X>(v, a, a, k, false);
+    if (FLB_TC_TRISQ) sqr_diag<X>(v, a); else blk_prod<X, X>(v, a, a, k, false);
     __syncwarp();  // every lane of the group has read its a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -534,7 +580,7 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
   const int k = threadIdx.x % 2;
   {
     uint32_t v[2 * X];
-    if (FLB_TC_TRISQ) sqr_local<X>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
+    if (FLB_TC_TRISQ) sqr_diag<X>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
     __syncwarp();  // both lanes have read a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
