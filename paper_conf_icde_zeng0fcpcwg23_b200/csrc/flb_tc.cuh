@@ -324,6 +324,9 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 #ifndef FLB_TC_TRISQ
 #define FLB_TC_TRISQ 1  // diagonal blocks a_k^2 as lane-local triangular squares (0: full X x X blk_prod)
 #endif
+#ifndef FLB_TC_TRISQ_EXP
+#define FLB_TC_TRISQ_EXP 2  // k_tc_exp (decryption; two-launch key-holder stages): the half-split form
+#endif
 
 // v = a^2 (2X words) for this lane's own block, X (X - 1) / 2 + X limb products instead of X^2
 // (squarings dominate the modexp).  U = sum_{i<j} a_i a_j 2^(32 (i + j)) by rows
@@ -414,9 +417,9 @@ __device__ __forceinline__ void sqr_local_split(uint32_t (&v)[2 * X], const uint
   asm volatile("addc.u32 %0, %0, 0;" : "+r"(v[2 * X - 1]));
 }
 
-template <int X>
+template <int X, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void sqr_diag(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
-  if constexpr (FLB_TC_TRISQ == 2) sqr_local_split<X>(v, a); else sqr_local<X>(v, a);
+  if constexpr (SQ == 2) sqr_local_split<X>(v, a); else sqr_local<X>(v, a);
 }
 
 // address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work row
@@ -504,7 +507,7 @@ __device__ __forceinline__ uint32_t add_sparse_chain(uint32_t (&q)[N], F add) {
 #endif
 }
 
-template <int S>
+template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
                                                   uint32_t* sW) {
   constexpr int X = Cfg<S>::X, H = X / 2;
@@ -513,7 +516,7 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
   {
     // diagonal block: t[2Xk, 2Xk + 2X) = a_k^2 (the four tile t exactly)
     uint32_t v[2 * X];
-    if (FLB_TC_TRISQ) sqr_diag<X>(v, a); else blk_prod<X, X>(v, a, a, k, false);
+    if (SQ) sqr_diag<X, SQ>(v, a); else blk_prod<X, X>(v, a, a, k, false);
     __syncwarp();  // every lane of the group has read its a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -573,14 +576,14 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
 // t[2Xk, 2Xk + 2X)) and half of the cross block, a_0 a_1[H k, + H) (X x H, doubled, added at words
 // X + H k), 384 instead of 512 limb products per lane.  The two cross pieces overlap, so they are
 // added in two phases; both carries land in lane 1's half and are folded in by lane 1.
-template <int S>
+template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
                                                      uint32_t* sW) {
   constexpr int X = Cfg<S>::X, H = X / 2;
   const int k = threadIdx.x % 2;
   {
     uint32_t v[2 * X];
-    if (FLB_TC_TRISQ) sqr_diag<X>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
+    if (SQ) sqr_diag<X, SQ>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
     __syncwarp();  // both lanes have read a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -847,7 +850,7 @@ __device__ __forceinline__ void tc_general_product(const uint32_t (&a)[Cfg<S>::X
 // The product phase of tc_mont: t = a b (2S words) for the 128 elements of the tile, t_lo into the
 // elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of T lanes per element
 // (X = 16 limbs each), NP passes of EP elements.  CTA-collective (no trailing barrier).
-template <int S>
+template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq, uint8_t* sA, uint32_t* sW) {
   using C = Cfg<S>;
   constexpr int X = C::X, KCH = C::KCH;
@@ -862,7 +865,7 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
 #if FLB_TC_SQR32
     if constexpr (FLB_TC_SQR && T == 2) {
       if (sq) {
-        tc_square_product_t2<S>(a, elem, sA, sW);
+        tc_square_product_t2<S, SQ>(a, elem, sA, sW);
         continue;
       }
     }
@@ -873,7 +876,7 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
           __syncwarp();  // a may come from the work row the quarters are stored into
           tc_square_product_reg<S>(a, elem, sA, sW);
         } else {
-          tc_square_product<S>(a, elem, sA, sW);
+          tc_square_product<S, SQ>(a, elem, sA, sW);
         }
         continue;
       }
@@ -928,7 +931,7 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
 
 // Montgomery product over the tile: for every element, a b R^-1 mod N (canonical) into its work
 // row.  sq: b = a.  `phase` tracks the mbarrier parity (two completions per call).  CTA-collective.
-template <int S>
+template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, const Smem& sm,
                                         const uint32_t* __restrict__ Nmod, uint32_t& phase) {
   using C = Cfg<S>;
@@ -939,7 +942,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
 #if FLB_TC_PROF
   long long t_ = clock64();
 #endif
-  tc_product<S>(sa, sb, sq, sA, sW);
+  tc_product<S, SQ>(sa, sb, sq, sA, sW);
   fence_async_smem();
   tc_before_sync();
   __syncthreads();
@@ -1303,7 +1306,7 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
 // One tile (128 elements) of problem P: the element powers x^E (or (1 + m n) x^E) into P.out.  `tab`
 // is the CTA's window-table scratch ([entry][kTileM][S] words).  The Toeplitz operands of P are in
 // shared memory (tc_load_operands).
-template <int S>
+template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, const uint32_t* one, uint32_t* tab,
                                             const Smem& sm, uint32_t& phase) {
   const Src row = src_row();
@@ -1314,21 +1317,21 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
   const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
   const uint32_t* xb = P.x + e0 * P.x_stride;
   if (P.x_words <= (uint32_t)S) {
-    tc_mont<S>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
   } else {
-    tc_mont<S>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
     tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
-    tc_mont<S>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
+    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
                phase);                                      // hi R^2
     tc_row_add<S>(sm, slot(0), P.N);
   }
   tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
   if (TB > 1) {
-    tc_mont<S>(row, row, true, sm, P.N, phase);             // x^2
+    tc_mont<S, SQ>(row, row, true, sm, P.N, phase);             // x^2
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
 #pragma unroll 1
     for (int t = 1; t < TB; t++) {
-      tc_mont<S>(slot(t - 1), slot(TB), false, sm, P.N, phase);
+      tc_mont<S, SQ>(slot(t - 1), slot(TB), false, sm, P.N, phase);
       tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
     }
   }
@@ -1340,21 +1343,21 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
     const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
 #pragma unroll 1
     for (int t = 0; t < sq; t++) {
-      tc_mont<S>(cur, cur, true, sm, P.N, phase);
+      tc_mont<S, SQ>(cur, cur, true, sm, P.N, phase);
       cur = row;
     }
     if (idx >= 0) {
-      tc_mont<S>(cur, slot(idx), false, sm, P.N, phase);
+      tc_mont<S, SQ>(cur, slot(idx), false, sm, P.N, phase);
       cur = row;
     }
   }
   if (P.m) {
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
-    tc_mont<S>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
+    tc_mont<S, SQ>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
     tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
-    tc_mont<S>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
+    tc_mont<S, SQ>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
   } else {
-    tc_mont<S>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
+    tc_mont<S, SQ>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
   }
   tc_row_store<S>(sm, P.out + e0 * S, S, nvalid);
 }
@@ -1407,7 +1410,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp(const ExpArgs A) {
       __syncthreads();
       loaded = pi;
     }
-    tc_exp_tile<S>(P, pi == 0 ? gt : gt - A.pb[0].tiles, A.one, tab, sm, phase);
+    tc_exp_tile<S, FLB_TC_TRISQ_EXP>(P, pi == 0 ? gt : gt - A.pb[0].tiles, A.one, tab, sm, phase);
     __syncthreads();  // the work rows are rewritten by the next tile's first product
   }
   tc_cta_fini<C::TMEM_COLS>(tmem_sh);
