@@ -324,6 +324,9 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 #ifndef FLB_TC_TRISQ
 #define FLB_TC_TRISQ 1  // diagonal blocks a_k^2 as lane-local triangular squares (0: full X x X blk_prod)
 #endif
+#ifndef FLB_TC_TRISQ_S1
+#define FLB_TC_TRISQ_S1 2  // stage-1 tiles (S = 32) of k_tc_exp_dag: the half-split form
+#endif
 #ifndef FLB_TC_TRISQ_EXP
 #define FLB_TC_TRISQ_EXP 2  // k_tc_exp (decryption; two-launch key-holder stages): the half-split form
 #endif
@@ -1468,7 +1471,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, co
       __syncthreads();
       tc_exp_tile<S2>(P, tile, A2.one, tab, sm, phase);
     } else {
-      tc_exp_tile<S1>(P, tile, A1.one, tab, sm, phase);
+      tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm, phase);
     }
     __syncthreads();  // the tile's output rows are stored; the work rows are rewritten next
     if (threadIdx.x == 0) {
