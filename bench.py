@@ -388,8 +388,7 @@ def run_flb(args):
             enc_kernel = ("k_tc_exp<32> + k_tc_exp<64> (two-stage key-holder encryption; Montgomery reduction as "
                           "u8 tcgen05 MMAs, t = a b on the IMAD pipe)")
         else:
-            enc_kernel = ("k_encrypt_crt<16,4>" if os.environ.get("FLB_CRT_V1") == "1"
-                          else "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)")
+            enc_kernel = "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)"
     else:
         enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
         enc_kernel = "k_encrypt<16,8>"

@@ -25,6 +25,13 @@
  *    scalar_mul and reduce return the mathematical function of the given integers; decrypt is
  *    specified for units c of Z_{n^2} (every unit is a valid ciphertext) and its
  *    output for a non-unit is unspecified.
+ *  - FLB_DEBUG_CHECKS=1 in the environment (read per call) turns on device-side range checks
+ *    before the op: plaintexts m < n (encrypt, encrypt_crt), ciphertexts c < n^2 (decrypt, add,
+ *    scalar_mul, reduce_segments, multiexp_segments; the modulus for flb_mod_*), offsets well
+ *    formed and idx in [0, num_inputs) (reduce_segments, multiexp_segments), per-plaintext
+ *    summands <= 2^pad_bits (unpack).  The call then synchronises `stream` and returns
+ *    FLB_EINVAL naming the violation and the number of offending elements.  gcd(r, n) = 1 is
+ *    not checked (probability of a violation ~2^(1-k/2), reading c4).
  */
 #ifndef FLB_PAILLIER_H
 #define FLB_PAILLIER_H
@@ -160,7 +167,10 @@ int flb_pack(const flb_pub* pub, const flb_codec* codec, const float* x, size_t 
 
 /* Unpack + dequantise (reading c14): x_i = Sum_i / sigma - cnt * alpha in binary64,
  * rounded to float32, with cnt = summands[i / slots] (device uint32 [num_pt]) or
- * summands_scalar when summands is NULL.  Errors: FLB_EINVAL, FLB_ECUDA. */
+ * summands_scalar when summands is NULL.  cnt <= 2^pad_bits: the b = pad_bits overflow bits of a
+ * slot hold at most 2^b summands "so that no overflow or inconsistent decryption results occur"
+ * (reading c15).  Errors: FLB_EINVAL (also summands_scalar > 2^pad_bits; a device
+ * array is checked only under FLB_DEBUG_CHECKS), FLB_ECUDA. */
 int flb_unpack(const flb_pub* pub, const flb_codec* codec, const uint32_t* pt, size_t n_values,
                const uint32_t* summands, uint32_t summands_scalar, float* x, void* stream);
 

@@ -30,15 +30,26 @@ library_path = _lib.LIB_PATH
 
 
 def _stream(stream: Optional[torch.cuda.Stream] = None) -> ctypes.c_void_p:
+    """The launch stream: `stream`, else the current stream of the CURRENT device — callers run
+    inside ``_on(tensor)``, which makes the tensors' device current (the library launches on and
+    uploads key constants to the current device)."""
     s = stream if stream is not None else torch.cuda.current_stream()
     return ctypes.c_void_p(s.cuda_stream)
+
+
+def _on(t: torch.Tensor):
+    """Make t's device the current CUDA device for the duration of a library call."""
+    return torch.cuda.device(t.device)
 
 
 def _ptr(t: Optional[torch.Tensor]) -> Optional[int]:
     return None if t is None else t.data_ptr()
 
 
-def _check_batch(t: torch.Tensor, words: int, name: str) -> int:
+def _check_batch(t: torch.Tensor, words: int, name: str, rows: Optional[int] = None,
+                 like: Optional[torch.Tensor] = None) -> int:
+    """Validate a [count, words] limb batch; ``rows``: required row count (an output buffer or a
+    second operand); ``like``: must live on the same device."""
     if not t.is_cuda:
         raise ValueError("%s must be a CUDA tensor" % name)
     if t.dtype not in (torch.int32, torch.uint32):
@@ -47,7 +58,20 @@ def _check_batch(t: torch.Tensor, words: int, name: str) -> int:
         raise ValueError("%s must be a contiguous [count, %d] tensor, got %s" % (name, words, tuple(t.shape)))
     if t.data_ptr() % 16:
         raise ValueError("%s must be 16-byte aligned" % name)
+    if rows is not None and t.shape[0] != rows:
+        raise ValueError("%s must have %d rows, got %d" % (name, rows, t.shape[0]))
+    if like is not None and t.device != like.device:
+        raise ValueError("%s is on %s, expected %s" % (name, t.device, like.device))
     return t.shape[0]
+
+
+def _check_vec(t: torch.Tensor, dtypes, name: str, min_len: int, like: torch.Tensor) -> None:
+    if not t.is_cuda or t.dtype not in dtypes or t.dim() != 1 or not t.is_contiguous():
+        raise ValueError("%s must be a contiguous CUDA %s vector" % (name, "/".join(str(d) for d in dtypes)))
+    if t.shape[0] < min_len:
+        raise ValueError("%s must have at least %d entries, got %d" % (name, min_len, t.shape[0]))
+    if t.device != like.device:
+        raise ValueError("%s is on %s, expected %s" % (name, t.device, like.device))
 
 
 def _limbs_of(x: int, words: int):
@@ -129,11 +153,13 @@ def miller_rabin(cand: torch.Tensor, rounds: int, mont_bases: Optional[torch.Ten
     words = cand.shape[1]
     M = _check_batch(cand, words, "cand")
     if mont_bases is not None:
-        _check_batch(mont_bases, words, "mont_bases")
+        _check_batch(mont_bases, words, "mont_bases", rows=M * rounds, like=cand)
     if out is None:
         out = torch.empty((M,), dtype=torch.int32, device=cand.device)
-    check("flb_miller_rabin", LIB.flb_miller_rabin(_ptr(cand), words, _ptr(mont_bases), rounds,
-                                                   seed & 0xFFFFFFFFFFFFFFFF, _ptr(out), M, _stream(stream)))
+    _check_vec(out, (torch.int32, torch.uint32), "out", M, cand)
+    with _on(cand):
+        check("flb_miller_rabin", LIB.flb_miller_rabin(_ptr(cand), words, _ptr(mont_bases), rounds,
+                                                       seed & 0xFFFFFFFFFFFFFFFF, _ptr(out), M, _stream(stream)))
     return out
 
 
@@ -152,12 +178,13 @@ def encrypt(pub: PublicKey, m: torch.Tensor, r: Optional[torch.Tensor] = None, s
     """Paillier::encrypt (PAPER L253, Eq. 3): c = (1 + m n) r^n mod n^2; r = Philox(seed, ctr0 + i) if None."""
     M = _check_batch(m, pub.pt_words, "m")
     if r is not None:
-        _check_batch(r, pub.pt_words, "r")
+        _check_batch(r, pub.pt_words, "r", rows=M, like=m)
     if out is None:
         out = torch.empty((M, pub.ct_words), dtype=torch.int32, device=m.device)
-    _check_batch(out, pub.ct_words, "out")
-    check("flb_encrypt", LIB.flb_encrypt(pub.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0, _ptr(out), M,
-                                         _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=M, like=m)
+    with _on(m):
+        check("flb_encrypt", LIB.flb_encrypt(pub.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0, _ptr(out),
+                                             M, _stream(stream)))
     return out
 
 
@@ -167,12 +194,13 @@ def encrypt_crt(priv: PrivateKey, m: torch.Tensor, r: Optional[torch.Tensor] = N
     pub = priv.pub
     M = _check_batch(m, pub.pt_words, "m")
     if r is not None:
-        _check_batch(r, pub.pt_words, "r")
+        _check_batch(r, pub.pt_words, "r", rows=M, like=m)
     if out is None:
         out = torch.empty((M, pub.ct_words), dtype=torch.int32, device=m.device)
-    _check_batch(out, pub.ct_words, "out")
-    check("flb_encrypt_crt", LIB.flb_encrypt_crt(priv.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0,
-                                                 _ptr(out), M, _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=M, like=m)
+    with _on(m):
+        check("flb_encrypt_crt", LIB.flb_encrypt_crt(priv.handle, _ptr(m), _ptr(r), seed & 0xFFFFFFFFFFFFFFFF, ctr0,
+                                                     _ptr(out), M, _stream(stream)))
     return out
 
 
@@ -182,8 +210,9 @@ def decrypt(priv: PrivateKey, c: torch.Tensor, out: Optional[torch.Tensor] = Non
     M = _check_batch(c, pub.ct_words, "c")
     if out is None:
         out = torch.empty((M, pub.pt_words), dtype=torch.int32, device=c.device)
-    _check_batch(out, pub.pt_words, "out")
-    check("flb_decrypt", LIB.flb_decrypt(priv.handle, _ptr(c), _ptr(out), M, _stream(stream)))
+    _check_batch(out, pub.pt_words, "out", rows=M, like=c)
+    with _on(c):
+        check("flb_decrypt", LIB.flb_decrypt(priv.handle, _ptr(c), _ptr(out), M, _stream(stream)))
     return out
 
 
@@ -191,12 +220,12 @@ def add(pub: PublicKey, c1: torch.Tensor, c2: torch.Tensor, out: Optional[torch.
         stream=None) -> torch.Tensor:
     """Paillier::add (PAPER L255, Eq. 5): c1 c2 mod n^2."""
     M = _check_batch(c1, pub.ct_words, "c1")
-    if _check_batch(c2, pub.ct_words, "c2") != M:
-        raise ValueError("c1 and c2 differ in count")
+    _check_batch(c2, pub.ct_words, "c2", rows=M, like=c1)
     if out is None:
         out = torch.empty_like(c1)
-    _check_batch(out, pub.ct_words, "out")
-    check("flb_add", LIB.flb_add(pub.handle, _ptr(c1), _ptr(c2), _ptr(out), M, _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=M, like=c1)
+    with _on(c1):
+        check("flb_add", LIB.flb_add(pub.handle, _ptr(c1), _ptr(c2), _ptr(out), M, _stream(stream)))
     return out
 
 
@@ -204,14 +233,15 @@ def scalar_mul(pub: PublicKey, c: torch.Tensor, e: torch.Tensor, out: Optional[t
                stream=None) -> torch.Tensor:
     """c^e mod n^2 = E(e m) (mod_pow); e: [count, e_words] unsigned limbs."""
     M = _check_batch(c, pub.ct_words, "c")
-    if e.dim() != 2 or e.shape[0] != M:
+    if e.dim() != 2:
         raise ValueError("e must be [count, e_words]")
-    _check_batch(e, e.shape[1], "e")
+    _check_batch(e, e.shape[1], "e", rows=M, like=c)
     if out is None:
         out = torch.empty_like(c)
-    _check_batch(out, pub.ct_words, "out")
-    check("flb_scalar_mul", LIB.flb_scalar_mul(pub.handle, _ptr(c), _ptr(e), e.shape[1], _ptr(out), M,
-                                               _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=M, like=c)
+    with _on(c):
+        check("flb_scalar_mul", LIB.flb_scalar_mul(pub.handle, _ptr(c), _ptr(e), e.shape[1], _ptr(out), M,
+                                                   _stream(stream)))
     return out
 
 
@@ -219,17 +249,17 @@ def reduce_segments(pub: PublicKey, c: torch.Tensor, offsets: torch.Tensor, idx:
                     max_segment_len: int = 0, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
     """out[j] = prod_{t in [off[j], off[j+1])} c[idx[t]] mod n^2 (empty = 1)."""
     L = _check_batch(c, pub.ct_words, "c")
-    if offsets.dtype != torch.int64 or not offsets.is_cuda or offsets.dim() != 1 or not offsets.is_contiguous():
-        raise ValueError("offsets must be a contiguous CUDA int64 vector")
+    _check_vec(offsets, (torch.int64,), "offsets", 1, c)
     S = offsets.shape[0] - 1
-    if idx is not None and (idx.dtype != torch.int64 or not idx.is_cuda or not idx.is_contiguous()):
-        raise ValueError("idx must be a contiguous CUDA int64 vector")
+    if idx is not None:
+        _check_vec(idx, (torch.int64,), "idx", 0, c)
     if out is None:
         out = torch.empty((S, pub.ct_words), dtype=torch.int32, device=c.device)
-    _check_batch(out, pub.ct_words, "out")
+    _check_batch(out, pub.ct_words, "out", rows=S, like=c)
     nent = idx.shape[0] if idx is not None else L
-    check("flb_reduce_segments", LIB.flb_reduce_segments(pub.handle, _ptr(c), L, _ptr(idx), nent, _ptr(offsets), S,
-                                                         max_segment_len, _ptr(out), _stream(stream)))
+    with _on(c):
+        check("flb_reduce_segments", LIB.flb_reduce_segments(pub.handle, _ptr(c), L, _ptr(idx), nent, _ptr(offsets),
+                                                             S, max_segment_len, _ptr(out), _stream(stream)))
     return out
 
 
@@ -237,18 +267,23 @@ def multiexp_segments(pub: PublicKey, c: torch.Tensor, e: torch.Tensor, offsets:
                       idx: Optional[torch.Tensor] = None, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
     """out[j] = prod_{t in seg j} c[idx[t]]^(e[t]) mod n^2 (per-entry exponents e [entries, e_words])."""
     L = _check_batch(c, pub.ct_words, "c")
-    if offsets.dtype != torch.int64 or not offsets.is_cuda or offsets.dim() != 1 or not offsets.is_contiguous():
-        raise ValueError("offsets must be a contiguous CUDA int64 vector")
+    _check_vec(offsets, (torch.int64,), "offsets", 1, c)
     S = offsets.shape[0] - 1
+    if e.dim() != 2:
+        raise ValueError("e must be [entries, e_words]")
     nent = e.shape[0]
-    _check_batch(e, e.shape[1], "e")
-    if idx is not None and (idx.dtype != torch.int64 or not idx.is_cuda or not idx.is_contiguous()):
-        raise ValueError("idx must be a contiguous CUDA int64 vector")
+    _check_batch(e, e.shape[1], "e", like=c)
+    if idx is not None:
+        _check_vec(idx, (torch.int64,), "idx", nent, c)
+    elif nent > L:
+        raise ValueError("without idx, e must have at most as many rows as c")
     if out is None:
         out = torch.empty((S, pub.ct_words), dtype=torch.int32, device=c.device)
-    _check_batch(out, pub.ct_words, "out")
-    check("flb_multiexp_segments", LIB.flb_multiexp_segments(pub.handle, _ptr(c), L, _ptr(idx), _ptr(e), e.shape[1],
-                                                             _ptr(offsets), S, nent, _ptr(out), _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=S, like=c)
+    with _on(c):
+        check("flb_multiexp_segments", LIB.flb_multiexp_segments(pub.handle, _ptr(c), L, _ptr(idx), _ptr(e),
+                                                                 e.shape[1], _ptr(offsets), S, nent, _ptr(out),
+                                                                 _stream(stream)))
     return out
 
 
@@ -274,39 +309,48 @@ def pack(pub: PublicKey, codec: Codec, x: torch.Tensor, out: Optional[torch.Tens
     M = codec.num_plaintexts(x.shape[0])
     if out is None:
         out = torch.empty((M, pub.pt_words), dtype=torch.int32, device=x.device)
-    _check_batch(out, pub.pt_words, "out")
+    _check_batch(out, pub.pt_words, "out", rows=M, like=x)
     cs = codec.struct()
-    check("flb_pack", LIB.flb_pack(pub.handle, ctypes.byref(cs), _ptr(x), x.shape[0], _ptr(out), _stream(stream)))
+    with _on(x):
+        check("flb_pack", LIB.flb_pack(pub.handle, ctypes.byref(cs), _ptr(x), x.shape[0], _ptr(out),
+                                       _stream(stream)))
     return out
 
 
 def unpack(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int,
            summands: Union[int, torch.Tensor] = 1, out: Optional[torch.Tensor] = None, stream=None) -> torch.Tensor:
     """Unpack + dequantise: x = Sum/sigma - cnt*alpha (float64 -> float32)."""
-    _check_batch(pt, pub.pt_words, "pt")
+    npt = codec.num_plaintexts(n_values)
+    if _check_batch(pt, pub.pt_words, "pt") < npt:
+        raise ValueError("pt must have at least %d rows for %d values" % (npt, n_values))
     if out is None:
         out = torch.empty((n_values,), dtype=torch.float32, device=pt.device)
+    _check_vec(out, (torch.float32,), "out", n_values, pt)
     cs = codec.struct()
     if isinstance(summands, torch.Tensor):
-        if summands.dtype not in (torch.int32, torch.uint32) or not summands.is_cuda:
-            raise ValueError("summands must be a CUDA int32 vector")
+        _check_vec(summands, (torch.int32, torch.uint32), "summands", npt, pt)
         sp, ss = _ptr(summands), 0
     else:
         sp, ss = None, int(summands)
-    check("flb_unpack", LIB.flb_unpack(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, sp, ss, _ptr(out),
-                                       _stream(stream)))
+    with _on(pt):
+        check("flb_unpack", LIB.flb_unpack(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, sp, ss, _ptr(out),
+                                           _stream(stream)))
     return out
 
 
 def unpack_sums(pub: PublicKey, codec: Codec, pt: torch.Tensor, n_values: int, out: Optional[torch.Tensor] = None,
                 stream=None) -> torch.Tensor:
     """The exact slot integers (int64 view of uint64)."""
-    _check_batch(pt, pub.pt_words, "pt")
+    npt = codec.num_plaintexts(n_values)
+    if _check_batch(pt, pub.pt_words, "pt") < npt:
+        raise ValueError("pt must have at least %d rows for %d values" % (npt, n_values))
     if out is None:
         out = torch.empty((n_values,), dtype=torch.int64, device=pt.device)
+    _check_vec(out, (torch.int64,), "out", n_values, pt)
     cs = codec.struct()
-    check("flb_unpack_sums", LIB.flb_unpack_sums(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, _ptr(out),
-                                                 _stream(stream)))
+    with _on(pt):
+        check("flb_unpack_sums", LIB.flb_unpack_sums(pub.handle, ctypes.byref(cs), _ptr(pt), n_values, _ptr(out),
+                                                     _stream(stream)))
     return out
 
 
@@ -328,18 +372,24 @@ class Modulus:
 
     def mul(self, a: torch.Tensor, b: torch.Tensor, out=None, stream=None) -> torch.Tensor:
         M = _check_batch(a, self.words, "a")
-        _check_batch(b, self.words, "b")
+        _check_batch(b, self.words, "b", rows=M, like=a)
         out = torch.empty_like(a) if out is None else out
-        check("flb_mod_mul", LIB.flb_mod_mul(self._h, _ptr(a), _ptr(b), _ptr(out), M, _stream(stream)))
+        _check_batch(out, self.words, "out", rows=M, like=a)
+        with _on(a):
+            check("flb_mod_mul", LIB.flb_mod_mul(self._h, _ptr(a), _ptr(b), _ptr(out), M, _stream(stream)))
         return out
 
     def pow(self, base: torch.Tensor, e: torch.Tensor, out=None, stream=None) -> torch.Tensor:
         """Per-element exponents e [count, e_words] (device)."""
         M = _check_batch(base, self.words, "base")
-        _check_batch(e, e.shape[1], "e")
+        if e.dim() != 2:
+            raise ValueError("e must be [count, e_words]")
+        _check_batch(e, e.shape[1], "e", rows=M, like=base)
         out = torch.empty_like(base) if out is None else out
-        check("flb_mod_pow", LIB.flb_mod_pow(self._h, _ptr(base), _ptr(e), e.shape[1], _ptr(out), M,
-                                             _stream(stream)))
+        _check_batch(out, self.words, "out", rows=M, like=base)
+        with _on(base):
+            check("flb_mod_pow", LIB.flb_mod_pow(self._h, _ptr(base), _ptr(e), e.shape[1], _ptr(out), M,
+                                                 _stream(stream)))
         return out
 
     def pow_shared(self, base: torch.Tensor, e: int, out=None, stream=None) -> torch.Tensor:
@@ -347,8 +397,10 @@ class Modulus:
         M = _check_batch(base, self.words, "base")
         ew = max(1, (e.bit_length() + 31) // 32)
         out = torch.empty_like(base) if out is None else out
-        check("flb_mod_pow_shared", LIB.flb_mod_pow_shared(self._h, _ptr(base), _limbs_of(e, ew), ew, _ptr(out), M,
-                                                           _stream(stream)))
+        _check_batch(out, self.words, "out", rows=M, like=base)
+        with _on(base):
+            check("flb_mod_pow_shared", LIB.flb_mod_pow_shared(self._h, _ptr(base), _limbs_of(e, ew), ew, _ptr(out),
+                                                               M, _stream(stream)))
         return out
 
 
@@ -455,12 +507,15 @@ def op_cost(key, op: str) -> Tuple[int, int]:
 
 def debug_tc_product(a: torch.Tensor, b: torch.Tensor, square: bool = False, stream=None) -> torch.Tensor:
     """The tensor-core Montgomery kernel's product phase alone: a_i b_i (or a_i^2) as 2w-limb rows,
-    w = a.shape[1] in {32, 64}, at most 128 rows (debugging and parity tests)."""
+    w = a.shape[1] in {32, 64}, at most 128 rows (debugging and parity tests).  square: 0/False =
+    general product, 1/True = block squaring (one triangular diagonal square per lane), 2 = block
+    squaring with the half-split diagonal square."""
     M = _check_batch(a, a.shape[1], "a")
-    _check_batch(b, a.shape[1], "b")
+    _check_batch(b, a.shape[1], "b", rows=M, like=a)
     out = torch.empty((M, 2 * a.shape[1]), dtype=torch.int32, device=a.device)
-    check("flb_debug_tc_product", LIB.flb_debug_tc_product(_ptr(a), _ptr(b), _ptr(out), M, a.shape[1], int(square),
-                                                           _stream(stream)))
+    with _on(a):
+        check("flb_debug_tc_product", LIB.flb_debug_tc_product(_ptr(a), _ptr(b), _ptr(out), M, a.shape[1],
+                                                               int(square), _stream(stream)))
     return out
 
 
@@ -468,8 +523,11 @@ def debug_mont_mul(pub: PublicKey, a: torch.Tensor, b: torch.Tensor, out: Option
                    stream=None) -> torch.Tensor:
     """a b R^-1 mod n^2 (the Montgomery primitive of PAPER Alg. 2)."""
     M = _check_batch(a, pub.ct_words, "a")
-    _check_batch(b, pub.ct_words, "b")
+    _check_batch(b, pub.ct_words, "b", rows=M, like=a)
     if out is None:
         out = torch.empty_like(a)
-    check("flb_debug_mont_mul", LIB.flb_debug_mont_mul(pub.handle, _ptr(a), _ptr(b), _ptr(out), M, _stream(stream)))
+    _check_batch(out, pub.ct_words, "out", rows=M, like=a)
+    with _on(a):
+        check("flb_debug_mont_mul", LIB.flb_debug_mont_mul(pub.handle, _ptr(a), _ptr(b), _ptr(out), M,
+                                                           _stream(stream)))
     return out

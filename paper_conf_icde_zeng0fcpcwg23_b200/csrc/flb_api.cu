@@ -24,6 +24,7 @@ flb_pub* make_pub(const Limbs& n_in) {
   K->n2_n0inv = C.n0inv;
   K->enc = H::best_schedule(K->n, 7);
   K->o_n2 = K->blob.put(K->n2, K->s);
+  K->o_n = K->blob.put(K->n, K->sp);
   K->o_R2 = K->blob.put(C.R2, K->s);
   K->o_R1 = K->blob.put(C.R1, K->s);
   K->o_nR = K->blob.put(C.to(K->n), K->s);
@@ -246,24 +247,17 @@ static uint64_t sched_squarings(const H::Schedule& S) {
 }
 
 // IMAD-pipe limb products of the tensor-core kernel (flb_tc.cuh) for `mults` S-word Montgomery
-// products of which `sqr` are squarings: S^2 for the row-scan product; for the block squaring
-// (S >= 64 on 4 lanes, S = 32 on 2) S (S + 1) / 2 with triangular diagonal blocks (FLB_TC_TRISQ),
-// else 10 (S/4)^2 on 4 lanes, 3 (S/2)^2 on 2
+// products of which `sqr` are squarings: S^2 for the row-scan product, S (S + 1) / 2 for the block
+// squaring with triangular diagonal blocks
 static uint64_t tc_imad_lp(uint64_t S, uint64_t mults, uint64_t sqr) {
-  const bool blk = FLB_TC_SQR && (S >= 64 || FLB_TC_SQR32);
-  const uint64_t sq_lp = !blk           ? S * S
-                         : FLB_TC_TRISQ ? S * (S + 1) / 2
-                         : S >= 64      ? 10 * (S / 4) * (S / 4)
-                                        : 3 * (S / 2) * (S / 2);
-  return (mults - sqr) * S * S + sqr * sq_lp;
+  return (mults - sqr) * S * S + sqr * (S * (S + 1) / 2);
 }
 
 // u8 MACs the two Toeplitz MMAs of one S-word tensor-core Montgomery product issue per element (MMA
 // row): K-slices of 32 bytes, q = t N' mod R over columns [32 ks, KB), q N over [0, min(KB, 32 ks + 48))
-// (flb_tc.cuh mma_toeplitz_lo / _hi; 2 KB^2 with FLB_TC_TRI=0)
+// (flb_tc.cuh mma_toeplitz_lo / _hi)
 static uint64_t tc_mma_macs(uint64_t S) {
   const uint64_t KB = 4 * S;
-  if (!FLB_TC_TRI) return 2 * KB * KB;
   uint64_t m = 0;
   for (uint64_t ks = 0; ks < KB / 32; ks++) m += 32 * (KB - 32 * ks) + 32 * std::min<uint64_t>(KB, 32 * ks + 48);
   return m;
@@ -294,8 +288,7 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
     }
     case 4: {  // key-holder encryption
       if (!V) return fail(FLB_EINVAL, "key-holder cost needs the private key");
-      const char* v1 = getenv("FLB_CRT_V1");
-      if (V->H && !(v1 && atoi(v1) == 1)) {
+      if (V->H) {
         // v2: per prime, stage 1 at the half frame (2 entry + table + schedule(Q) + exit) and stage 2
         // at sp (entry + table + schedule(P) + m n + final); CRT 1 + plain product
         const uint64_t h = V->H, ch = 2 * h * h + h;
@@ -433,6 +426,58 @@ uint32_t flb_slot_capacity(const flb_pub* K, uint32_t slot_bits) {
   return (K && slot_bits) ? (K->nbits - 1) / slot_bits : 0;
 }
 
+}  // extern "C"
+
+// ----------------------------------------------------------------------------- FLB_DEBUG_CHECKS
+// With FLB_DEBUG_CHECKS=1 in the environment (read per call) the batch calls first run range-check
+// kernels over their inputs (m < n, c < n^2, idx / offsets well formed, summands <= 2^pad_bits),
+// wait for them and return FLB_EINVAL naming the violation; off (the default) the hot path checks
+// nothing beyond the synchronous argument checks (include/flb_paillier.h).
+static int dbg_grid(uint64_t n) { return (int)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 4096)); }
+static bool debug_checks() {
+  const char* e = getenv("FLB_DEBUG_CHECKS");
+  return e && atoi(e) != 0;
+}
+template <typename F>
+static int run_check(cudaStream_t st, const std::string& what, F launch) {
+  unsigned long long* d = nullptr;
+  unsigned long long h = 0;
+  FLB_CK(cudaMallocAsync(&d, sizeof(h), st));
+  FLB_CK(cudaMemsetAsync(d, 0, sizeof(h), st));
+  launch(d);
+  cudaError_t e = cudaGetLastError();
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, st);
+  cudaFreeAsync(d, st);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return fail(FLB_ECUDA, std::string("FLB_DEBUG_CHECKS: ") + cudaGetErrorString(e));
+  if (h) return fail(FLB_EINVAL, "FLB_DEBUG_CHECKS: " + std::to_string(h) + " " + what);
+  return FLB_OK;
+}
+// rows x_i ([count][words], contiguous) must be < bound (device, words limbs)
+static int check_below(const uint32_t* x, uint64_t count, uint32_t words, const uint32_t* bound, void* stream,
+                       const char* what) {
+  cudaStream_t st = (cudaStream_t)stream;
+  return run_check(st, what, [&](unsigned long long* d) {
+    flb::k_check_below<<<dbg_grid(count), 256, 0, st>>>(x, count, words, bound, words, d);
+  });
+}
+static int check_segments(const int64_t* idx, size_t num_entries, size_t num_inputs, const int64_t* offsets,
+                          size_t num_segments, void* stream) {
+  cudaStream_t st = (cudaStream_t)stream;
+  int rc = run_check(st, "malformed offsets (offsets[0] = 0, non-decreasing, offsets[S] = num_entries)",
+                     [&](unsigned long long* d) {
+                       flb::k_check_offsets<<<dbg_grid(num_segments + 1), 256, 0, st>>>(offsets, num_segments,
+                                                                                     (int64_t)num_entries, d);
+                     });
+  if (rc || !idx || num_entries == 0) return rc;
+  return run_check(st, "idx entries outside [0, num_inputs)", [&](unsigned long long* d) {
+    flb::k_check_index<<<dbg_grid(num_entries), 256, 0, st>>>(idx, num_entries, (int64_t)num_inputs, d);
+  });
+}
+static int pub_dev(const flb_pub* K, uint32_t** dev) { return const_cast<DevBlob&>(K->dev).get(K->blob, dev); }
+
+extern "C" {
+
 int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* c,
                 size_t count, void* stream) {
   if (!K || !m || !c) return fail(FLB_EINVAL, "null pointer");
@@ -440,6 +485,7 @@ int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
+  if (debug_checks() && (rc = check_below(m, count, K->sp, dev + K->o_n, stream, "plaintexts m >= n"))) return rc;
   FLB_DISPATCH_ENC(K->frame, run_encrypt, K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 
@@ -463,6 +509,12 @@ int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count,
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
   if (rc) return rc;
+  if (debug_checks()) {
+    uint32_t* pd;
+    if ((rc = pub_dev(V->pub, &pd)) ||
+        (rc = check_below(c, count, V->pub->s, pd + V->pub->o_n2, stream, "ciphertexts c >= n^2")))
+      return rc;
+  }
   if (use_tc(V)) {
     if (V->pub->sp == 64) return run_decrypt_tc<64>(V, dev, c, m, count, (cudaStream_t)stream);
     return run_decrypt_tc<32>(V, dev, c, m, count, (cudaStream_t)stream);
@@ -480,8 +532,13 @@ int flb_encrypt_crt(const flb_priv* V, const uint32_t* m, const uint32_t* r, uin
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(V->dev).get(V->blob, &dev);
   if (rc) return rc;
-  const char* v1 = getenv("FLB_CRT_V1");
-  if (V->H && !(v1 && atoi(v1) == 1)) return encrypt_crt_v2(V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+  if (debug_checks()) {
+    uint32_t* pd;
+    if ((rc = pub_dev(V->pub, &pd)) ||
+        (rc = check_below(m, count, V->pub->sp, pd + V->pub->o_n, stream, "plaintexts m >= n")))
+      return rc;
+  }
+  if (V->H) return encrypt_crt_v2(V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
   FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt, V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 
@@ -491,6 +548,9 @@ int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* 
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
+  if (debug_checks() && ((rc = check_below(c1, count, K->s, dev + K->o_n2, stream, "c1 >= n^2")) ||
+                         (rc = check_below(c2, count, K->s, dev + K->o_n2, stream, "c2 >= n^2"))))
+    return rc;
   FLB_DISPATCH_ENC(K->frame, run_add_plain, K, dev, c1, c2, out, count, (cudaStream_t)stream);
 }
 
@@ -520,6 +580,7 @@ int flb_scalar_mul(const flb_pub* K, const uint32_t* c, const uint32_t* e, uint3
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
+  if (debug_checks() && (rc = check_below(c, count, K->s, dev + K->o_n2, stream, "ciphertexts c >= n^2"))) return rc;
   FLB_DISPATCH_ENC(K->frame, run_smul, K, dev, c, e, e_words, out, count, (cudaStream_t)stream);
 }
 
@@ -533,6 +594,10 @@ int flb_reduce_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs, 
   uint32_t* dev;
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
+  if (debug_checks() &&
+      ((rc = check_segments(idx, num_entries, num_inputs, offsets, num_segments, stream)) ||
+       (num_inputs && (rc = check_below(c, num_inputs, K->s, dev + K->o_n2, stream, "ciphertexts c >= n^2")))))
+    return rc;
   FLB_DISPATCH_ENC(K->frame, run_reduce, K, dev, c, num_entries, idx, offsets, num_segments, max_segment_len, out,
                    (cudaStream_t)stream);
 }
@@ -668,6 +733,13 @@ int flb_multiexp_segments(const flb_pub* K, const uint32_t* c, size_t num_inputs
   if (e_words < 1 || e_words > 8) return fail(FLB_EINVAL, "e_words must be in [1, 8]");
   if (num_segments == 0) return FLB_OK;
   cudaStream_t st = (cudaStream_t)stream;
+  if (debug_checks()) {
+    uint32_t* dev;
+    int rc;
+    if ((rc = pub_dev(K, &dev)) || (rc = check_segments(idx, num_entries, num_inputs, offsets, num_segments, stream)) ||
+        (num_inputs && (rc = check_below(c, num_inputs, K->s, dev + K->o_n2, stream, "ciphertexts c >= n^2"))))
+      return rc;
+  }
   const uint32_t s_words = K->s;
   const uint64_t Kb = 32ull * e_words;
   const uint64_t avg = num_entries / num_segments;
@@ -925,7 +997,18 @@ int flb_unpack(const flb_pub* K, const flb_codec* cd, const uint32_t* pt, size_t
   flb::CodecArgs A;
   int rc = codec_args(K, cd, &A);
   if (rc) return rc;
+  // the b = pad_bits overflow bits hold at most 2^b summands per slot
+  const uint64_t cap = cd->pad_bits >= 63 ? ~0ull : (1ull << cd->pad_bits);
+  if (!summands && (uint64_t)summands_scalar > cap) return fail(FLB_EINVAL, "summands > 2^pad_bits (slot overflow)");
   if (n_values == 0) return FLB_OK;
+  if (summands && debug_checks()) {
+    const uint64_t n_pt = (n_values + A.slots - 1) / A.slots;
+    cudaStream_t st = (cudaStream_t)stream;
+    rc = run_check(st, "summands > 2^pad_bits (slot overflow)", [&](unsigned long long* d) {
+      flb::k_check_counts<<<grid_1d(n_pt), 256, 0, st>>>(summands, n_pt, cap, d);
+    });
+    if (rc) return rc;
+  }
   flb::k_unpack<<<grid_1d(n_values), 256, 0, (cudaStream_t)stream>>>(pt, n_values, A, summands, summands_scalar, x);
   FLB_LAUNCH_CHECK();
   return FLB_OK;

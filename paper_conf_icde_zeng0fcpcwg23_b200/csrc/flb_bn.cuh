@@ -298,33 +298,12 @@ __device__ __forceinline__ void mont_mul(uint32_t (&r)[X], const uint32_t (&a)[X
   mont_mul_staged<X, T>(r, a, n, n0inv);
 }
 
-// r = a * a * R^-1 mod N
-template <int X, int T>
-__device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
-                                                uint32_t n0inv);
-
-template <int X, int T>
-__device__ __forceinline__ void mont_sqr_split(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
-                                               uint32_t n0inv);
-
-#ifndef FLB_SQR_BLOCKS
-#define FLB_SQR_BLOCKS 0  // measured slower on B200; kept as a parity-tested experiment
-#endif
-#ifndef FLB_SQR_SPLIT
-#define FLB_SQR_SPLIT 0  // bit-exact but measured slower on B200; parity-tested experiment
-#endif
 
 template <int X, int T>
 __device__ __forceinline__ void mont_sqr(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
                                          uint32_t n0inv) {
-  if constexpr (FLB_SQR_BLOCKS && T >= 4) {
-    mont_sqr_blocks<X, T>(r, a, n, n0inv);
-  } else if constexpr (FLB_SQR_SPLIT && T >= 2 && X >= 8 && X % 8 == 0) {
-    mont_sqr_split<X, T>(r, a, n, n0inv);
-  } else {
-    stage<X, T>(a);
-    mont_mul_staged<X, T>(r, a, n, n0inv);
-  }
+  stage<X, T>(a);
+  mont_mul_staged<X, T>(r, a, n, n0inv);
 }
 
 // r = a * b mod 2^(32*S) (the low half of the plain product).
@@ -446,125 +425,6 @@ __device__ __forceinline__ void redc_step(uint32_t (&E)[X + 1], uint32_t (&O)[X 
   for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
 }
 
-template <int X, int T>
-__device__ __forceinline__ void mont_sqr_blocks(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
-                                                uint32_t n0inv) {
-  constexpr int LD = X + 4, S = X * T, NB = T / 2 + 1;
-  static_assert(T >= 4, "block squaring needs at least 4 lanes per integer");
-  const int k = (int)(lane_id() & (T - 1));
-  stage<X, T>(a);
-  const uint32_t* bs = stage_group<X, T>();
-  unsigned long long* col = col_group<X, T>();
-#pragma unroll
-  for (int j = 0; j < 2 * X; j += 2)
-    *reinterpret_cast<ulonglong2*>(col + 2 * X * k + j) = make_ulonglong2(0ull, 0ull);
-  __syncwarp();
-#pragma unroll 1
-  for (int blk = 0; blk < NB; blk++) {
-    const int l = (k + blk) & (T - 1);
-    const bool active = (blk < T / 2) || (k < T / 2);
-    const bool wraps = (k + blk) >= T;
-    const unsigned long long f = blk == 0 ? 1ull : 2ull;
-    const uint32_t* row = bs + l * LD;
-    uint32_t E[X + 1], O[X + 1], pend = 0, lo[X], hi[X];
-#pragma unroll
-    for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
-#pragma unroll
-    for (int jj = 0; jj < X; jj++) lo[jj] = local_row<X>(E, O, pend, a, row[jj]);
-    // the high X words (the block product is < 2^(64 X): nothing above)
-    asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(hi[0]) : "r"(E[0]), "r"(pend));
-#pragma unroll
-    for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(hi[t]) : "r"(E[t]), "r"(O[t - 1]));
-    unsigned long long* cb = col + X * (k + l);
-    // f * (lo, hi) into the column sums: batches of 8 columns, all loads of a batch before its
-    // stores (ptxas would otherwise serialise each load behind the previous store)
-    const unsigned sh = blk == 0 ? 0u : 1u;
-#pragma unroll
-    for (int ph = 0; ph < 2; ph++) {
-      if (active && (wraps == (ph == 1))) {
-#pragma unroll
-        for (int j0 = 0; j0 < 2 * X; j0 += 8) {
-          ulonglong2 v[4];
-#pragma unroll
-          for (int u = 0; u < 4; u++) v[u] = *reinterpret_cast<const ulonglong2*>(cb + j0 + 2 * u);
-#pragma unroll
-          for (int u = 0; u < 4; u++) {
-            const int j = j0 + 2 * u;
-            const uint32_t w0 = j < X ? lo[j] : hi[j - X], w1 = j + 1 < X ? lo[j + 1] : hi[j + 1 - X];
-            v[u].x += (unsigned long long)w0 << sh;
-            v[u].y += (unsigned long long)w1 << sh;
-          }
-#pragma unroll
-          for (int u = 0; u < 4; u++) *reinterpret_cast<ulonglong2*>(cb + j0 + 2 * u) = v[u];
-        }
-      }
-      __syncwarp();
-    }
-    (void)f;
-  }
-  // normalise lane k's two chunks: lo = columns [kX, kX+X), hi = [S + kX, S + kX + X)
-  uint32_t tl[X], th[X];
-  unsigned long long cl = 0, ch = 0;
-  {
-    const unsigned long long* pl = col + X * k;
-    const unsigned long long* ph = col + S + X * k;
-#pragma unroll
-    for (int j = 0; j < X; j++) {
-      cl += pl[j];
-      tl[j] = (uint32_t)cl;
-      cl >>= 32;
-      ch += ph[j];
-      th[j] = (uint32_t)ch;
-      ch >>= 32;
-    }
-  }
-  // chunk chain lo_0 .. lo_{T-1}, hi_0 .. hi_{T-1}: pass each chunk's carry to the next chunk
-  uint32_t inl_lo = __shfl_up_sync(FULL, (uint32_t)cl, 1, T), inl_hi = __shfl_up_sync(FULL, (uint32_t)(cl >> 32), 1, T);
-  uint32_t inh_lo = __shfl_up_sync(FULL, (uint32_t)ch, 1, T), inh_hi = __shfl_up_sync(FULL, (uint32_t)(ch >> 32), 1, T);
-  const uint32_t top_lo = __shfl_sync(FULL, (uint32_t)cl, T - 1, T), top_hi = __shfl_sync(FULL, (uint32_t)(cl >> 32), T - 1, T);
-  if (k == 0) {
-    inl_lo = 0; inl_hi = 0;
-    inh_lo = top_lo; inh_hi = top_hi;
-  }
-  uint32_t gl, gh;
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(tl[0]) : "r"(inl_lo));
-  asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(tl[1]) : "r"(inl_hi));
-#pragma unroll
-  for (int t = 2; t < X; t++) asm volatile("addc.cc.u32 %0, %0, 0;" : "+r"(tl[t]));
-  asm volatile("addc.u32 %0, 0, 0;" : "=r"(gl));
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(th[0]) : "r"(inh_lo));
-  asm volatile("addc.cc.u32 %0, %0, %1;" : "+r"(th[1]) : "r"(inh_hi));
-#pragma unroll
-  for (int t = 2; t < X; t++) asm volatile("addc.cc.u32 %0, %0, 0;" : "+r"(th[t]));
-  asm volatile("addc.u32 %0, 0, 0;" : "=r"(gh));
-  {
-    // single-bit carries along the 2T-chunk chain (lookahead over both ballots)
-    const uint32_t GL = __ballot_sync(FULL, gl != 0), PL = __ballot_sync(FULL, all_ones<X>(tl));
-    const uint32_t GH = __ballot_sync(FULL, gh != 0), PH = __ballot_sync(FULL, all_ones<X>(th));
-    const int base = (T == 32) ? 0 : (int)(lane_id() & ~(uint32_t)(T - 1));
-    const uint64_t mask = (T == 32) ? 0xffffffffull : ((1ull << T) - 1);
-    const uint64_t gg = (((uint64_t)GL >> base) & mask) | ((((uint64_t)GH >> base) & mask) << T);
-    const uint64_t pp = (((uint64_t)PL >> base) & mask) | ((((uint64_t)PH >> base) & mask) << T);
-    const uint64_t c = ((pp | gg) + gg) ^ pp;
-    add_word_propagate<X>(tl, (uint32_t)((c >> k) & 1u));
-    add_word_propagate<X>(th, (uint32_t)((c >> (T + k)) & 1u));
-  }
-  // REDC(t_lo) + t_hi
-  uint32_t E[X + 1], O[X + 1], pend = 0;
-#pragma unroll
-  for (int t = 0; t < X; t++) { E[t] = tl[t]; O[t] = 0; }
-  E[X] = 0;
-  O[X] = 0;
-#pragma unroll 1
-  for (int kk = 0; kk < T; kk++) {
-#pragma unroll
-    for (int jj = 0; jj < X; jj++) redc_step<X, T>(E, O, pend, n, n0inv);
-  }
-  const uint32_t over1 = collapse<X, T>(r, E, O, pend);
-  const uint32_t over2 = grp_add<X, T>(r, r, th);
-  grp_cond_sub<X, T>(r, n, over1 | over2);
-}
-
 // ----------------------------------------------------------------------------- split squaring
 // Montgomery squaring with a quarter of the square's limb products moved out of the reduced part.
 // With B = 2^(32 S/2), R = B^2 and a = L + H B (L, H the low / high halves of a):
@@ -632,87 +492,6 @@ __device__ __forceinline__ uint32_t prod_step(uint32_t (&E)[HX + 1], uint32_t (&
 #pragma unroll
   for (int t = 0; t <= HX; t++) { E[t] = nE[t]; O[t] = nO[t]; }
   return out;
-}
-
-template <int X, int T>
-__device__ __forceinline__ void mont_sqr_split(uint32_t (&r)[X], const uint32_t (&a)[X], const uint32_t (&n)[X],
-                                               uint32_t n0inv) {
-  constexpr int LD = X + 4, HX = X / 2, T2 = T / 2;
-  const int k = (int)(lane_id() & (T - 1));
-  stage<X, T>(a);
-  uint32_t* bs = stage_group<X, T>();
-  // a'' = L + 2 H B: lanes >= T/2 hold 2H (bits shifted up across lanes, none into lane T/2);
-  // the top bit of 2H is added as b_i * tb at word S (lane T-1, word X) in every phase-1 step
-  uint32_t ad[X];
-  {
-    uint32_t cin = __shfl_up_sync(FULL, a[X - 1], 1, T) >> 31;
-    if (k == T2) cin = 0;
-    const bool upper = k >= T2;
-#pragma unroll
-    for (int j = X - 1; j >= 1; j--) ad[j] = upper ? __funnelshift_l(a[j - 1], a[j], 1) : a[j];
-    ad[0] = upper ? ((a[0] << 1) | cin) : a[0];
-  }
-  const uint32_t tb = __shfl_sync(FULL, a[X - 1], T - 1, T) >> 31;
-  const uint32_t tmask = (tb != 0 && k == T - 1) ? 0xffffffffu : 0u;
-  uint32_t E[X + 1], O[X + 1], pend = 0;
-#pragma unroll
-  for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
-  // phase 1: multiplier words L_0 .. L_{S/2-1}
-#pragma unroll 1
-  for (int kk = 0; kk < T2; kk++) {
-    const uint32_t* row = bs + kk * LD;
-#pragma unroll
-    for (int jj = 0; jj < X; jj++) {
-      const uint32_t bi = row[jj];
-      cios_step_top<X, T>(E, O, pend, ad, bi, bi & tmask, n, n0inv);
-    }
-  }
-  // H spread over all T lanes: lane k holds H words [k HX, (k+1) HX) = staged row T/2 + k/2
-  uint32_t hl[HX];
-  {
-    const uint4* q = reinterpret_cast<const uint4*>(bs + (T2 + (k >> 1)) * LD + (k & 1) * HX);
-#pragma unroll
-    for (int v = 0; v < HX / 4; v++) {
-      const uint4 u = q[v];
-      hl[4 * v] = u.x; hl[4 * v + 1] = u.y; hl[4 * v + 2] = u.z; hl[4 * v + 3] = u.w;
-    }
-  }
-  __syncwarp();  // the L rows are dead from here on: phase 2 writes H^2's low words there
-  uint32_t E2[HX + 1], O2[HX + 1], pend2 = 0;
-#pragma unroll
-  for (int t = 0; t <= HX; t++) { E2[t] = 0; O2[t] = 0; }
-  // phase 2: reduce-only steps, each with one row of H^2 (multiplier word H_j = staged word S/2 + j)
-#pragma unroll 1
-  for (int kk = T2; kk < T; kk++) {
-    const uint32_t* row = bs + kk * LD;
-    uint32_t* outrow = bs + (kk - T2) * LD;
-#pragma unroll
-    for (int jj = 0; jj < X; jj++) {
-      const uint32_t hj = row[jj];
-      redc_step<X, T>(E, O, pend, n, n0inv);
-      const uint32_t w = prod_step<HX, T>(E2, O2, pend2, hl, hj);
-      if (k == 0) outrow[jj] = w;  // H^2 word (kk - T/2) X + jj
-    }
-  }
-  uint32_t over = collapse<X, T>(r, E, O, pend);
-  uint32_t h2[X];
-  {
-    uint32_t hh[HX];
-    collapse<HX, T>(hh, E2, O2, pend2);  // H^2 words S/2 + k HX ..; H^2 < R, no overflow
-    __syncwarp();                         // every lane has read its last H row
-    uint4* q = reinterpret_cast<uint4*>(bs + (T2 + (k >> 1)) * LD + (k & 1) * HX);
-#pragma unroll
-    for (int v = 0; v < HX / 4; v++) q[v] = make_uint4(hh[4 * v], hh[4 * v + 1], hh[4 * v + 2], hh[4 * v + 3]);
-    __syncwarp();
-    const uint4* p = reinterpret_cast<const uint4*>(bs + k * LD);
-#pragma unroll
-    for (int v = 0; v < X / 4; v++) {
-      const uint4 u = p[v];
-      h2[4 * v] = u.x; h2[4 * v + 1] = u.y; h2[4 * v + 2] = u.z; h2[4 * v + 3] = u.w;
-    }
-  }
-  over |= grp_add<X, T>(r, r, h2);
-  grp_cond_sub<X, T>(r, n, over);
 }
 
 // ----------------------------------------------------------------------------- loads / stores

@@ -110,7 +110,7 @@ struct flb_pub {
   uint32_t n2_n0inv = 0;
   H::Schedule enc;
   Blob blob;
-  size_t o_n2 = 0, o_R2 = 0, o_R1 = 0, o_nR = 0, o_RL = 0, o_sched = 0;
+  size_t o_n2 = 0, o_n = 0, o_R2 = 0, o_R1 = 0, o_nR = 0, o_RL = 0, o_sched = 0;
   DevBlob dev;
 };
 
@@ -208,17 +208,8 @@ inline int resident_blocks(K kernel, int* blocks) {
   return FLB_OK;
 }
 
-// Grid for `items` work units of T lanes each: at most the resident capacity; the units are then
-// spread evenly over the rounds the persistent loop needs (ceil(items / capacity)), so the last
-// round is not a sliver of the grid — only with FLB_BALANCE=1: measured slower on B200 (fewer
-// resident warps cost more than the partial last round).
-inline bool balance_rounds() {
-  static bool v = [] {
-    const char* e = getenv("FLB_BALANCE");
-    return e && atoi(e) == 1;
-  }();
-  return v;
-}
+// Grid for `items` work units of T lanes each: at most the resident capacity (the persistent loop
+// takes the rest; balancing the rounds was measured slower on B200).
 
 template <int T, typename K>
 inline int grid_for(K kernel, uint64_t items, int* grid) {
@@ -227,14 +218,7 @@ inline int grid_for(K kernel, uint64_t items, int* grid) {
   if (rc) return rc;
   const uint64_t per_block = kBlock / T;  // work units per block
   const uint64_t cap_items = (uint64_t)cap * per_block;
-  uint64_t want = items;
-  if (items > cap_items) {
-    want = cap_items;
-    if (balance_rounds()) {
-      const uint64_t rounds = (items + cap_items - 1) / cap_items;
-      want = (items + rounds - 1) / rounds;
-    }
-  }
+  const uint64_t want = std::min(items, cap_items);
   *grid = (int)std::max<uint64_t>(1, (want + per_block - 1) / per_block);
   return FLB_OK;
 }
@@ -603,8 +587,17 @@ int launch_tc_exp_dag(flb::tc::ExpArgs& A1, flb::tc::ExpArgs& A2, cudaStream_t s
 template <int S>
 int run_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, int sq, cudaStream_t st) {
   using C = flb::tc::Cfg<S>;
-  FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM));
-  flb::tc::k_tc_debug_product<S><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, sq);
+  // sq: 0 = general product, 1 = block squaring with one triangular diagonal square per lane,
+  // 2 = the half-split diagonal square (the form k_tc_exp and stage 1 of k_tc_exp_dag use)
+  if (sq == 2) {
+    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                C::SMEM));
+    flb::tc::k_tc_debug_product<S, 2><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, 1);
+  } else {
+    FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                C::SMEM));
+    flb::tc::k_tc_debug_product<S, 1><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, sq);
+  }
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }

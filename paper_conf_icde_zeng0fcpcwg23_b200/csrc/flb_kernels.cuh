@@ -400,6 +400,43 @@ static __global__ void k_fill_one(uint32_t* out, uint64_t count, uint32_t S) {
     out[i] = (i % S) == 0 ? 1u : 0u;
 }
 
+// ----------------------------------------------------------------------------- FLB_DEBUG_CHECKS
+// Value-range checks the hot path does not make (include/flb_paillier.h): each
+// counts the offending elements into *bad (one thread per element; debug mode only).
+// rows x_i (words limbs, row stride `stride`) with x_i >= bound
+static __global__ void k_check_below(const uint32_t* x, uint64_t count, uint32_t stride, const uint32_t* bound,
+                                     uint32_t words, unsigned long long* bad) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t* r = x + i * stride;
+    int c = 0;
+    for (int w = (int)words - 1; w >= 0 && c == 0; w--) {
+      const uint32_t a = r[w], b = __ldg(bound + w);
+      c = a < b ? -1 : a > b ? 1 : 0;
+    }
+    if (c >= 0) atomicAdd(bad, 1ull);
+  }
+}
+// int64 indices outside [0, hi)
+static __global__ void k_check_index(const int64_t* idx, uint64_t count, int64_t hi, unsigned long long* bad) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x) {
+    const int64_t v = idx[i];
+    if (v < 0 || v >= hi) atomicAdd(bad, 1ull);
+  }
+}
+// CSR offsets [segments + 1]: offsets[0] = 0, non-decreasing, offsets[segments] = total
+static __global__ void k_check_offsets(const int64_t* off, uint64_t segments, int64_t total, unsigned long long* bad) {
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j <= segments; j += (uint64_t)gridDim.x * blockDim.x) {
+    const int64_t v = off[j];
+    const bool ok = (j == 0 ? v == 0 : v >= off[j - 1]) && (j < segments || v == total);
+    if (!ok) atomicAdd(bad, 1ull);
+  }
+}
+// per-plaintext summand counts above the padding capacity 2^pad_bits (b overflow bits)
+static __global__ void k_check_counts(const uint32_t* cnt, uint64_t count, uint64_t limit, unsigned long long* bad) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < count; i += (uint64_t)gridDim.x * blockDim.x)
+    if ((uint64_t)cnt[i] > limit) atomicAdd(bad, 1ull);
+}
+
 // ----------------------------------------------------------------------------- Miller–Rabin (keygen)
 struct MrArgs {
   const uint32_t* cand;       // [count][S] odd candidates >= 5

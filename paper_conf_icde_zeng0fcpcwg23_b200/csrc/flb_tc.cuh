@@ -82,24 +82,6 @@ __device__ __forceinline__ uint32_t idesc_u8(int m, int n) {
   return (2u << 4) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
 }
 
-// D[tmem] = sum over the K-slices ks of A[:, 32 ks ..] x B_ks^T, B_ks the 8-row-aligned window of the
-// extended operand starting at row r0 - 32 ks
-__device__ __forceinline__ void mma_toeplitz(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext, uint32_t r0,
-                                             uint32_t idesc) {
-  for (uint32_t ks = 0; ks < kch / 2; ks++) {
-    const uint64_t ad = smem_desc(sa + ks * 256u, kch * 128u);
-    const uint64_t bd = smem_desc(ext + ((r0 - 32u * ks) >> 3) * 256u, 256u);
-    const uint32_t acc = ks > 0 ? 1u : 0u;
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-                 "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
-                 :: "r"(tmem_d), "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
-  }
-}
-
-#ifndef FLB_TC_TRI
-#define FLB_TC_TRI 1  // skip the all-zero (triangular) parts of the Toeplitz products (0: full N per K-slice)
-#endif
-
 // One K-slice MMA (A columns 32 ks .., B window starting at extended row r) into D columns [c0, c0 + n)
 __device__ __forceinline__ void mma_slice(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext, uint32_t ks,
                                           uint32_t r, uint32_t c0, uint32_t n, uint32_t acc) {
@@ -236,15 +218,45 @@ struct Smem {
 
 // An operand of tc_mont per element of the tile: the element's work row (row = true), or element j
 // of an array at p + j * stride with `words` limbs (the rest zero; elements >= `valid` read zeros;
-// stride 0 = one constant for all).
+// stride 0 = one constant for all).  `ld` says how the array may be read:
+//   kLdNC   ld.global.nc — kernel inputs and key constants, read-only for the whole launch;
+//   kLdCTA  plain ld.global — written earlier in the launch by this CTA and ordered by bar.sync
+//           (the window-table slots);
+//   kLdGPU  ld.relaxed.gpu — written by another CTA of this launch and published by the
+//           st.release / ld.acquire tile flag (stage-2 inputs of k_tc_exp_dag).
+enum : uint32_t { kLdNC = 0, kLdCTA = 1, kLdGPU = 2 };
 struct Src {
   const uint32_t* p;
   uint32_t stride, words, valid;
   bool row;
+  uint32_t ld;
 };
-__device__ __forceinline__ Src src_row() { return Src{nullptr, 0, 0, 0, true}; }
-__device__ __forceinline__ Src src_arr(const uint32_t* p, uint32_t stride, uint32_t words, uint32_t valid) {
-  return Src{p, stride, words, valid, false};
+__device__ __forceinline__ Src src_row() { return Src{nullptr, 0, 0, 0, true, kLdNC}; }
+__device__ __forceinline__ Src src_arr(const uint32_t* p, uint32_t stride, uint32_t words, uint32_t valid,
+                                       uint32_t ld = kLdNC) {
+  return Src{p, stride, words, valid, false, ld};
+}
+
+__device__ __forceinline__ uint4 ld_v4(const uint32_t* p, uint32_t ld) {
+  uint4 u;
+  if (ld == kLdGPU)
+    asm volatile("ld.relaxed.gpu.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(u.x), "=r"(u.y), "=r"(u.z), "=r"(u.w) : "l"(p) : "memory");
+  else if (ld == kLdCTA)
+    u = *reinterpret_cast<const uint4*>(p);
+  else
+    u = __ldg(reinterpret_cast<const uint4*>(p));
+  return u;
+}
+__device__ __forceinline__ uint32_t ld_u32(const uint32_t* p, uint32_t ld) {
+  uint32_t v;
+  if (ld == kLdGPU)
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  else if (ld == kLdCTA)
+    v = *p;
+  else
+    v = __ldg(p);
+  return v;
 }
 
 #ifndef FLB_TC_PROF
@@ -277,19 +289,22 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
       r[4 * v] = u.x; r[4 * v + 1] = u.y; r[4 * v + 2] = u.z; r[4 * v + 3] = u.w;
     }
   } else {
-    load_elem<C::X, C::T>(r, s.p + (size_t)elem * s.stride, s.words, (uint32_t)elem < s.valid);
+    // limbs [k X, k X + X) of the element (the rest of a short element reads zeros)
+    const uint32_t* base = s.p + (size_t)elem * s.stride;
+    const uint32_t w0 = (uint32_t)(k * C::X);
+    const bool valid = (uint32_t)elem < s.valid;
+    if (valid && w0 + C::X <= s.words) {
+#pragma unroll
+      for (int v = 0; v < C::X / 4; v++) {
+        const uint4 u = ld_v4(base + w0 + 4 * v, s.ld);
+        r[4 * v] = u.x; r[4 * v + 1] = u.y; r[4 * v + 2] = u.z; r[4 * v + 3] = u.w;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < C::X; j++) r[j] = (valid && w0 + j < s.words) ? ld_u32(base + w0 + j, s.ld) : 0u;
+    }
   }
 }
-
-#ifndef FLB_TC_SQR
-#define FLB_TC_SQR 1  // block squaring in the product phase (0: squarings use the general product)
-#endif
-#ifndef FLB_TC_CHAIN
-#define FLB_TC_CHAIN 1  // carry chains of the squaring's in-place additions as add.cc/addc.cc (0: 64-bit sums)
-#endif
-#ifndef FLB_TC_SQR32
-#define FLB_TC_SQR32 1  // block squaring also at S = 32 (two lanes per element)
-#endif
 
 // ----------------------------------------------------------------------------- squaring product
 // t = a^2 for the product phase when a = b (87 % of the multiplications of a modexp).  Lane k of the
@@ -322,7 +337,7 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 }
 
 #ifndef FLB_TC_TRISQ
-#define FLB_TC_TRISQ 1  // diagonal blocks a_k^2 as lane-local triangular squares (0: full X x X blk_prod)
+#define FLB_TC_TRISQ 1  // diagonal blocks a_k^2: 1 = one lane-local triangular square, 2 = the half-split form
 #endif
 #ifndef FLB_TC_TRISQ_S1
 #define FLB_TC_TRISQ_S1 2  // stage-1 tiles (S = 32) of k_tc_exp_dag: the half-split form
@@ -437,7 +452,6 @@ __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, i
 // chain (add.cc / addc.cc, one IADD3.X per word) across the chunks; the doubling is a funnel shift.
 template <int S, int NW, bool DBL = true>
 __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int elem, int w0, const uint32_t (&v)[NW]) {
-#if FLB_TC_CHAIN
   uint32_t prev = 0, cy;
 #pragma unroll
   for (int c = 0; c < NW / 4; c++) {
@@ -459,35 +473,12 @@ __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int ele
   }
   asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
   return cy + (DBL ? prev >> 31 : 0u);
-#else
-  uint64_t cy = 0;
-  uint32_t prev = 0;
-#pragma unroll
-  for (int c = 0; c < NW / 4; c++) {
-    uint4* p = t_chunk<S>(sA, sW, elem, w0 + 4 * c);
-    const uint4 m = *p;
-    uint32_t d[4], r[4];
-    const uint32_t mm[4] = {m.x, m.y, m.z, m.w};
-#pragma unroll
-    for (int u = 0; u < 4; u++) {
-      const uint32_t x = v[4 * c + u];
-      d[u] = DBL ? (x << 1) | (prev >> 31) : x;
-      prev = x;
-      const uint64_t s = (uint64_t)mm[u] + d[u] + cy;
-      r[u] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    *p = make_uint4(r[0], r[1], r[2], r[3]);
-  }
-  return (uint32_t)cy + (DBL ? prev >> 31 : 0u);
-#endif
 }
 
 // q[j0 .. N) += the small addends add(j) (each < 2^32, nonzero at a few positions) with one carry
 // chain; returns the carry out of q[N - 1]
 template <int N, int J0, typename F>
 __device__ __forceinline__ uint32_t add_sparse_chain(uint32_t (&q)[N], F add) {
-#if FLB_TC_CHAIN
   uint32_t cy;
 #pragma unroll
   for (int j = J0; j < N; j++) {
@@ -498,16 +489,6 @@ __device__ __forceinline__ uint32_t add_sparse_chain(uint32_t (&q)[N], F add) {
   }
   asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
   return cy;
-#else
-  uint64_t cy = 0;
-#pragma unroll
-  for (int j = J0; j < N; j++) {
-    const uint64_t s = (uint64_t)q[j] + add(j) + cy;
-    q[j] = (uint32_t)s;
-    cy = s >> 32;
-  }
-  return (uint32_t)cy;
-#endif
 }
 
 template <int S, int SQ = FLB_TC_TRISQ>
@@ -519,7 +500,7 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
   {
     // diagonal block: t[2Xk, 2Xk + 2X) = a_k^2 (the four tile t exactly)
     uint32_t v[2 * X];
-    if (SQ) sqr_diag<X, SQ>(v, a); else blk_prod<X, X>(v, a, a, k, false);
+    sqr_diag<X, SQ>(v, a);
     __syncwarp();  // every lane of the group has read its a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -586,7 +567,7 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
   const int k = threadIdx.x % 2;
   {
     uint32_t v[2 * X];
-    if (SQ) sqr_diag<X, SQ>(v, a); else blk_prod<X, X, 2>(v, a, a, k, false);
+    sqr_diag<X, SQ>(v, a);
     __syncwarp();  // both lanes have read a (it may come from the work row)
 #pragma unroll
     for (int c = 0; c < X / 2; c++)
@@ -622,233 +603,6 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
   __syncwarp();
 }
 
-// Block squaring with the pieces summed in registers (FLB_TC_SQR == 2): the same block products as
-// tc_square_product, but each lane accumulates its own quarter Q_k = t[2Xk, 2Xk + 2X) in registers,
-// the off-diagonal pieces (undoubled) arriving from the lanes that computed them by shuffle; the
-// diagonal block a_k^2 is folded in last as t_k = 2 acc + a_k^2, and the quarters' carries are
-// resolved by one shuffle round plus a ballot carry-lookahead.  Shared memory sees only the final
-// quarter stores (no read-modify-write of t).
-template <int S>
-__device__ __forceinline__ void tc_square_product_reg(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
-                                                      uint32_t* sW) {
-  constexpr int X = Cfg<S>::X, H = X / 2, Q = 2 * X;
-  const int k = threadIdx.x % kT;
-  uint32_t acc[Q];
-  uint32_t qc = 0;  // carries out of the quarter (weight 2^(32 Q)), of the undoubled off-diagonal sum
-  {
-    // half block of lane k: a_i a_(i+2)[H hh, + H), i = k & 1, hh = k >> 1, at words Q i + Q + H hh:
-    // lane 0 -> Q_1 [0, X + H), lane 2 -> Q_1 [H, Q), lane 1 -> Q_2 [0, X + H), lane 3 -> Q_2 [H, Q)
-    uint32_t v[X + H];
-    {
-      uint32_t M[X];
-      const int i = k & 1, hh = k >> 1;
-#pragma unroll
-      for (int j = 0; j < X; j++) M[j] = __shfl_sync(FULL, a[j], i, kT);
-      blk_prod<X, H>(v, M, a, i + 2, hh == 1);
-    }
-    const bool rcv = (k == 1 || k == 2);
-#pragma unroll
-    for (int w = 0; w < X + H; w++) {
-      const uint32_t x = __shfl_up_sync(FULL, v[w], 1, kT);  // lane 1 <- lane 0, lane 2 <- lane 1
-      acc[w] = rcv ? x : 0u;
-    }
-#pragma unroll
-    for (int w = X + H; w < Q; w++) acc[w] = 0;
-    uint64_t cy = 0;
-#pragma unroll
-    for (int w = 0; w < X + H; w++) {
-      const uint32_t y = __shfl_down_sync(FULL, v[w], 1, kT);  // lane 1 <- lane 2, lane 2 <- lane 3
-      const uint64_t s = (uint64_t)acc[H + w] + (rcv ? y : 0u) + cy;
-      acc[H + w] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    qc += (uint32_t)cy;
-  }
-  {
-    // full block F_k = a_k a_(k+1 mod 4) at words X (2k + 1) (lane 3: 3X): low half -> Q_k [X, Q)
-    // (lane 3's -> Q_1), high half -> Q_(k+1) [0, X) (lane 3's -> Q_2)
-    uint32_t v[Q];
-    blk_prod<X, X>(v, a, a, (k + 1) & (kT - 1), false);
-    uint64_t cy = 0;
-#pragma unroll
-    for (int j = 0; j < X; j++) {
-      const uint32_t r3 = __shfl_sync(FULL, v[j], kT - 1, kT);
-      const uint64_t s = (uint64_t)acc[X + j] + (k < kT - 1 ? v[j] : 0u) + (k == 1 ? r3 : 0u) + cy;
-      acc[X + j] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    qc += (uint32_t)cy;
-    cy = 0;
-#pragma unroll
-    for (int j = 0; j < X; j++) {
-      const uint32_t u = __shfl_up_sync(FULL, v[X + j], 1, kT);
-      const uint32_t r3 = __shfl_sync(FULL, v[X + j], kT - 1, kT);
-      const uint64_t s = (uint64_t)acc[j] + (k >= 1 ? u : 0u) + (k == 2 ? r3 : 0u) + cy;
-      acc[j] = (uint32_t)s;
-      cy = s >> 32;
-    }
-#pragma unroll
-    for (int j = X; j < Q; j++) {
-      const uint64_t s = (uint64_t)acc[j] + cy;
-      acc[j] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    qc += (uint32_t)cy;
-  }
-  uint32_t cq;
-  {
-    // diagonal: Q_k = 2 acc + a_k^2, the product's low words folded in as its rows emerge
-    uint32_t E[X + 1], O[X + 1], pend = 0;
-#pragma unroll
-    for (int t = 0; t <= X; t++) { E[t] = 0; O[t] = 0; }
-    uint64_t cy = 0;
-    uint32_t prev = 0;
-#pragma unroll
-    for (int j = 0; j < X; j++) {
-      const uint32_t o = local_row<X>(E, O, pend, a, a[j]);
-      const uint32_t d = (acc[j] << 1) | (prev >> 31);
-      prev = acc[j];
-      const uint64_t s = (uint64_t)d + o + cy;
-      acc[j] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    uint32_t hw[X];
-    asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(hw[0]) : "r"(E[0]), "r"(pend));
-#pragma unroll
-    for (int t = 1; t < X; t++) asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(hw[t]) : "r"(E[t]), "r"(O[t - 1]));
-#pragma unroll
-    for (int t = 0; t < X; t++) {
-      const uint32_t d = (acc[X + t] << 1) | (prev >> 31);
-      prev = acc[X + t];
-      const uint64_t s = (uint64_t)d + hw[t] + cy;
-      acc[X + t] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    cq = 2 * qc + (prev >> 31) + (uint32_t)cy;
-  }
-  // carries between quarters: Q_(k-1)'s carry-out into Q_k, then single-bit ripples by lookahead
-  {
-    uint32_t cin = __shfl_up_sync(FULL, cq, 1, kT);
-    if (k == 0) cin = 0;
-    uint64_t cy = cin;
-#pragma unroll
-    for (int j = 0; j < Q; j++) {
-      const uint64_t s = (uint64_t)acc[j] + cy;
-      acc[j] = (uint32_t)s;
-      cy = s >> 32;
-    }
-    const uint32_t c = group_carry<kT>(cy != 0, all_ones<Q>(acc), 0);
-    add_word_propagate<Q>(acc, c & 1u);
-  }
-#pragma unroll
-  for (int c = 0; c < X / 2; c++)
-    *t_chunk<S>(sA, sW, elem, Q * k + 4 * c) = make_uint4(acc[4 * c], acc[4 * c + 1], acc[4 * c + 2], acc[4 * c + 3]);
-}
-
-#ifndef FLB_TC_GBLK
-#define FLB_TC_GBLK 0  // general products as lane-local X x X blocks: bit-exact but 2.7 % slower (spills)
-#endif
-
-// t = a b for a != b by lane-local X x X block products (the general products of a modexp: window
-// table, multiply steps, epilogue).  Lane k holds a_k, b_k (X words each); in round d it computes
-// a_k b_((k+d) mod T) (rows of b by shuffle, one per row) and adds it at words X (k + (k+d) mod T).
-// T = 4: round 0 fills the four quarters t[2Xk, 2Xk + 2X); rounds 1, 3 cover [X, 3X), [3X, 5X),
-// [5X, 7X) plus a second [3X, 5X) piece (two phases each); round 2 covers [2X, 4X) and [4X, 6X) twice
-// (two phases).  T = 2: round 0 fills the halves, round 1 adds a_0 b_1 and a_1 b_0 at [X, 3X) (two
-// phases).  Each piece's carry-out (0/1) lands at a fixed word; one fold pass per quarter adds them,
-// its carries resolved by a ballot carry-lookahead.  T X^2 limb products per lane, as the row scan.
-template <int S>
-__device__ __forceinline__ void tc_general_product(const uint32_t (&a)[Cfg<S>::X], const uint32_t (&b)[Cfg<S>::X],
-                                                   int elem, uint8_t* sA, uint32_t* sW) {
-  constexpr int X = Cfg<S>::X, T = Cfg<S>::T;
-  const int k = threadIdx.x % T;
-  {
-    uint32_t v[2 * X];
-    blk_prod<X, X, T>(v, a, b, k, false);
-    __syncwarp();  // every lane has its a, b (they may come from the work row)
-#pragma unroll
-    for (int c = 0; c < X / 2; c++)
-      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
-  }
-  if constexpr (T == 2) {
-    uint32_t v[2 * X];
-    blk_prod<X, X, T>(v, a, b, k ^ 1, false);
-    uint32_t cx = 0;
-    __syncwarp();
-    if (k == 0) cx = t_add_dbl<S, 2 * X, false>(sA, sW, elem, X, v);
-    __syncwarp();
-    if (k == 1) cx = t_add_dbl<S, 2 * X, false>(sA, sW, elem, X, v);
-    __syncwarp();
-    const uint32_t c0 = __shfl_sync(FULL, cx, 0, 2);
-    if (k == 1) {  // both carries at word 3X = lane 1's relative X; no carry leaves t
-      uint32_t q[X];
-#pragma unroll
-      for (int c = 0; c < X / 4; c++) {
-        const uint4 u = *t_chunk<S>(sA, sW, elem, 3 * X + 4 * c);
-        q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
-      }
-      add_sparse_chain<X, 0>(q, [&](int j) { return j == 0 ? c0 + cx : 0u; });
-#pragma unroll
-      for (int c = 0; c < X / 4; c++)
-        *t_chunk<S>(sA, sW, elem, 3 * X + 4 * c) = make_uint4(q[4 * c], q[4 * c + 1], q[4 * c + 2], q[4 * c + 3]);
-    }
-    __syncwarp();
-  } else {
-    static_assert(T == 4, "block product on 2 or 4 lanes");
-    uint32_t c1 = 0, c2 = 0, c3 = 0;
-    {  // round 1: a_k b_(k+1): lanes 0-2 at X (2k + 1), lane 3 at 3X; carries at X (2k + 3), lane 3 at 5X
-      uint32_t v[2 * X];
-      blk_prod<X, X, T>(v, a, b, (k + 1) & 3, false);
-      const int w0 = X * (k < 3 ? 2 * k + 1 : 3);
-      __syncwarp();
-      if (k < 3) c1 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-      __syncwarp();
-      if (k == 3) c1 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-    }
-    {  // round 3: a_k b_(k-1): lanes 1-3 at X (2k - 1), lane 0 at 3X; carries at X (2k + 1), lane 0 at 5X
-      uint32_t v[2 * X];
-      blk_prod<X, X, T>(v, a, b, (k + 3) & 3, false);
-      const int w0 = X * (k > 0 ? 2 * k - 1 : 3);
-      __syncwarp();
-      if (k > 0) c3 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-      __syncwarp();
-      if (k == 0) c3 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-    }
-    {  // round 2: a_k b_(k+2): lanes 0, 2 at 2X, lanes 1, 3 at 4X; carries at 4X, 6X
-      uint32_t v[2 * X];
-      blk_prod<X, X, T>(v, a, b, (k + 2) & 3, false);
-      const int w0 = X * (2 + 2 * (k & 1));
-      __syncwarp();
-      if (k < 2) c2 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-      __syncwarp();
-      if (k >= 2) c2 = t_add_dbl<S, 2 * X, false>(sA, sW, elem, w0, v);
-      __syncwarp();
-    }
-    // carries into quarter k ([2Xk, 2Xk + 2X)), at relative 0 and X:
-    //   q1: X <- c1(0) + c3(1);  q2: 0 <- c2(0) + c2(2), X <- c1(1) + c1(3) + c3(2) + c3(0);
-    //   q3: 0 <- c2(1) + c2(3), X <- c1(2) + c3(3)
-    const uint32_t a0 = __shfl_sync(FULL, c1, 0, T), a1 = __shfl_sync(FULL, c1, 1, T);
-    const uint32_t a2 = __shfl_sync(FULL, c1, 2, T), a3 = __shfl_sync(FULL, c1, 3, T);
-    const uint32_t b0 = __shfl_sync(FULL, c3, 0, T), b1 = __shfl_sync(FULL, c3, 1, T);
-    const uint32_t b2 = __shfl_sync(FULL, c3, 2, T), b3 = __shfl_sync(FULL, c3, 3, T);
-    const uint32_t d0 = __shfl_sync(FULL, c2, 0, T), d1 = __shfl_sync(FULL, c2, 1, T);
-    const uint32_t d2 = __shfl_sync(FULL, c2, 2, T), d3 = __shfl_sync(FULL, c2, 3, T);
-    const uint32_t at0 = k == 2 ? d0 + d2 : k == 3 ? d1 + d3 : 0u;
-    const uint32_t atX = k == 1 ? a0 + b1 : k == 2 ? a1 + a3 + b2 + b0 : k == 3 ? a2 + b3 : 0u;
-    uint32_t q[2 * X];
-#pragma unroll
-    for (int c = 0; c < X / 2; c++) {
-      const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c);
-      q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
-    }
-    const uint32_t cy = add_sparse_chain<2 * X, 0>(q, [&](int j) { return j == 0 ? at0 : j == X ? atX : 0u; });
-    const uint32_t c = group_carry<T>(cy != 0, all_ones<2 * X>(q), 0);
-    add_word_propagate<2 * X>(q, c & 1u);
-#pragma unroll
-    for (int cc = 0; cc < X / 2; cc++)
-      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
-  }
-}
 
 // The product phase of tc_mont: t = a b (2S words) for the 128 elements of the tile, t_lo into the
 // elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of T lanes per element
@@ -865,35 +619,19 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
     const int elem = h * C::EP + tid / T;
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
-#if FLB_TC_SQR32
-    if constexpr (FLB_TC_SQR && T == 2) {
+    if constexpr (T == 2) {
       if (sq) {
         tc_square_product_t2<S, SQ>(a, elem, sA, sW);
         continue;
       }
-    }
-#endif
-    if constexpr (FLB_TC_SQR && S >= 64) {  // block squaring needs X x X blocks on 4 lanes
-      if (sq) {
-        if (FLB_TC_SQR == 2) {
-          __syncwarp();  // a may come from the work row the quarters are stored into
-          tc_square_product_reg<S>(a, elem, sA, sW);
-        } else {
-          tc_square_product<S, SQ>(a, elem, sA, sW);
-        }
-        continue;
-      }
-    }
-    if (sq) {
-#pragma unroll
-      for (int j = 0; j < X; j++) b[j] = a[j];
     } else {
-      src_load<S>(b, sb, elem, sW);
-      if constexpr (FLB_TC_GBLK) {
-        tc_general_product<S>(a, b, elem, sA, sW);
+      static_assert(S >= 64, "block squaring needs X x X blocks on 4 lanes");
+      if (sq) {
+        tc_square_product<S, SQ>(a, elem, sA, sW);
         continue;
       }
     }
+    src_load<S>(b, sb, elem, sW);
     // stage b in the element's sA row (natural byte order: word w at chunk w / 4)
     __syncwarp();
 #pragma unroll
@@ -953,11 +691,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- M1: q columns [0, KB)
   if (tid == 0) {
     tc_after_sync();
-#if FLB_TC_TRI
     mma_toeplitz_lo(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E1));
-#else
-    mma_toeplitz(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E1), KB, idesc_u8(kTileM, KB));
-#endif
     mma_commit(sm.mbar);
   }
   // normalisation: TMEM lane quadrant L = warp % 4 (elements 32L ..), column half g = warp / 4
@@ -973,19 +707,10 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   TC_MARK(1);
   uint32_t v[QW];
   auto add_in = [&](uint64_t cin) {
-#if FLB_TC_CHAIN
     v[0] = add_cc(v[0], (uint32_t)cin);
     v[1] = addc_cc(v[1], (uint32_t)(cin >> 32));
 #pragma unroll
     for (int w = 2; w < QW; w++) v[w] = addc_cc(v[w], 0u);
-#else
-#pragma unroll
-    for (int w = 0; w < QW; w++) {
-      const uint64_t s = (uint64_t)v[w] + cin;
-      v[w] = (uint32_t)s;
-      cin = s >> 32;
-    }
-#endif
   };
   auto publish = [&](uint64_t carry) {
     uint32_t ao = 0xffffffffu;
@@ -1001,7 +726,6 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   };
   // ---- N1: q = D1 mod R
   {
-#if FLB_TC_CHAIN
     uint32_t hprev = 0;
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
@@ -1011,22 +735,6 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       norm8_chain<false>(cv, nullptr, v + c0 / 4, hprev, c0 == 0);
     }
     publish(addc_end(hprev, 0u));
-#else
-    uint64_t carry = 0;
-#pragma unroll
-    for (int c0 = 0; c0 < QC; c0 += 32) {
-      uint32_t cv[32];
-      tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
-      tmem_wait();
-#pragma unroll
-      for (int w = 0; w < 8; w++) {
-        const uint64_t s = carry + word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]);
-        v[c0 / 4 + w] = (uint32_t)s;
-        carry = s >> 32;
-      }
-    }
-    publish(carry);
-#endif
   }
   tc_before_sync();
   __syncthreads();  // D1 drained, t_lo bytes read, carries published
@@ -1040,11 +748,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- M2: q N columns [KB-8, 2KB-8) into D2 = TMEM [0, KB)
   if (tid == 0) {
     tc_after_sync();
-#if FLB_TC_TRI
     mma_toeplitz_hi(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E2));
-#else
-    mma_toeplitz(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E2), 2 * KB - 8, idesc_u8(kTileM, KB));
-#endif
     mma_commit(sm.mbar);
   }
   TC_MARK(2);
@@ -1065,9 +769,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       const uint64_t s1 = (s0 >> 32) + word_of(bc[4], bc[5], bc[6], bc[7]) + ttop.y;
       carry = (s1 >> 32) + ((((uint32_t)s0) | ((uint32_t)s1)) != 0u ? 1u : 0u);
     }
-#if FLB_TC_CHAIN
     uint32_t hprev = (uint32_t)carry;  // < 2^20
-#endif
     // this half's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; half 1's last 8 columns
     // (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
     uint32_t top[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -1109,22 +811,9 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       const uint4 h0 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[0];
       const uint4 h1 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[1];
       const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
-#if FLB_TC_CHAIN
       norm8_chain<true>(cv, th, v + c0 / 4, hprev, c0 == 0);
-#else
-#pragma unroll
-      for (int w = 0; w < 8; w++) {
-        const uint64_t s = carry + word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]) + th[w];
-        v[c0 / 4 + w] = (uint32_t)s;
-        carry = s >> 32;
-      }
-#endif
     }
-#if FLB_TC_CHAIN
     publish(addc_end(hprev, 0u));
-#else
-    publish(carry);
-#endif
   }
   tc_before_sync();
   __syncthreads();
@@ -1135,7 +824,6 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   uint32_t d[QW];
   {
     uint32_t br = 0, nzd = 0;
-#if FLB_TC_CHAIN
     uint32_t nn[QW];
 #pragma unroll
     for (int c = 0; c < QW / 4; c++) {
@@ -1148,20 +836,6 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     br = subc_end(0u, 0u) & 1u;
 #pragma unroll
     for (int w = 0; w < QW; w++) nzd |= d[w];
-#else
-#pragma unroll
-    for (int c = 0; c < QW / 4; c++) {
-      const uint4 nv = __ldg(reinterpret_cast<const uint4*>(Nmod + g * QW + 4 * c));
-      const uint32_t nn[4] = {nv.x, nv.y, nv.z, nv.w};
-#pragma unroll
-      for (int w = 0; w < 4; w++) {
-        const uint64_t df = (uint64_t)v[4 * c + w] - nn[w] - br;
-        d[4 * c + w] = (uint32_t)df;
-        br = (uint32_t)(df >> 63);
-        nzd |= (uint32_t)df;
-      }
-    }
-#endif
     xch[g].w = br | (nzd == 0u ? 2u : 0u);
   }
   __syncthreads();
@@ -1170,19 +844,9 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     const uint32_t b1 = f0 & 1u;                          // borrow into half 1
     const uint32_t bout = (f1 & 1u) | ((f1 >> 1) & b1);    // borrow out of the top
     if (ovf != 0 || bout == 0) {                           // u >= N: take u - N
-#if FLB_TC_CHAIN
       v[0] = sub_cc(d[0], g == 1 ? b1 : 0u);
 #pragma unroll
       for (int w = 1; w < QW; w++) v[w] = subc_cc(d[w], 0u);
-#else
-      uint32_t br = g == 1 ? b1 : 0u;
-#pragma unroll
-      for (int w = 0; w < QW; w++) {
-        const uint64_t df = (uint64_t)d[w] - br;
-        v[w] = (uint32_t)df;
-        br = (uint32_t)(df >> 63);
-      }
-#endif
     }
 #pragma unroll
     for (int c = 0; c < QW / 4; c++)
@@ -1311,20 +975,21 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
 // shared memory (tc_load_operands).
 template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, const uint32_t* one, uint32_t* tab,
-                                            const Smem& sm, uint32_t& phase) {
+                                            const Smem& sm, uint32_t& phase, uint32_t x_ld = kLdNC) {
   const Src row = src_row();
   const int TB = P.table;
-  auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM); };
+  auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM, kLdCTA); };
   auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
   const uint64_t e0 = tile * kTileM;
   const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
   const uint32_t* xb = P.x + e0 * P.x_stride;
   if (P.x_words <= (uint32_t)S) {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid, x_ld), src_arr(P.R2, 0, S, kTileM), false, sm, P.N,
+                   phase);
   } else {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid, x_ld), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
     tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
-    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
+    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid, x_ld), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
                phase);                                      // hi R^2
     tc_row_add<S>(sm, slot(0), P.N);
   }
@@ -1469,7 +1134,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, co
         }
       }
       __syncthreads();
-      tc_exp_tile<S2>(P, tile, A2.one, tab, sm, phase);
+      tc_exp_tile<S2>(P, tile, A2.one, tab, sm, phase, kLdGPU);  // y: written by another CTA of this launch
     } else {
       tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm, phase);
     }
@@ -1487,14 +1152,14 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, co
 }
 
 // debug: the product phase alone (t = a b, or a^2 when sq) for up to 128 elements -> t [count][2S]
-template <int S>
+template <int S, int SQ>
 __global__ void __launch_bounds__(kThreads, 1) k_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t,
                                                                   uint32_t count, int sq) {
   using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
   uint8_t* sA = smem + C::OFF_A;
   uint32_t* sW = reinterpret_cast<uint32_t*>(smem + C::OFF_W);
-  tc_product<S>(src_arr(a, S, S, count), src_arr(b, S, S, count), sq != 0, sA, sW);
+  tc_product<S, SQ>(src_arr(a, S, S, count), src_arr(b, S, S, count), sq != 0, sA, sW);
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < count * 2 * S; i += kThreads) {
     const uint32_t e = i / (2 * S), w = i % (2 * S);

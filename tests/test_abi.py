@@ -111,6 +111,11 @@ def test_batch_calls_validate_before_launch():
         cs = _lib.CodecStruct(a, qb, pb, sb, sl)
         assert L.flb_pack(pub.handle, ctypes.byref(cs), 16, 10, 16, None) == -1
         assert L.flb_unpack(pub.handle, ctypes.byref(cs), 16, 10, None, 1, 16, None) == -1
+    # b = pad_bits overflow bits hold at most 2^b summands per slot
+    cs = _lib.CodecStruct(1.0, 29, 3, 32, 31)
+    assert L.flb_unpack(pub.handle, ctypes.byref(cs), 16, 10, None, 9, 16, None) == -1
+    assert "2^pad_bits" in L.flb_last_error().decode()
+    assert L.flb_unpack(pub.handle, ctypes.byref(cs), 16, 0, None, 8, 16, None) == 0  # 8 = 2^3 is allowed
 
 
 def _sliding_mults(e, w):

@@ -21,14 +21,14 @@ pytestmark = pytest.mark.gpu
 KEYS = golden_keys()
 
 # (key, alpha, qbits, pad_bits, slots): C1 (L432 setting, S = 1), C2 (S = 63), C4 (w = 64, S = 2),
-# full 32-bit capacity at 1024 bits, toy key with a single slot
+# full 32-bit capacity at 1024 bits, full capacity at 3072 bits
 CASES = [
     ("1024", 0.5, 30, 2, 1),
     ("2048", 1.0, 29, 3, 63),
     ("2048", 1.0, 44, 20, 2),
     ("1024", 1.0, 29, 3, 31),
     ("4096", 1.0, 30, 34, 63),
-    ("toy16", 0.5, 8, 24, 0),
+    ("3072", 1.0, 29, 3, 95),
 ]
 
 
@@ -43,10 +43,6 @@ def test_pack_unpack(case):
     name, alpha, qb, pb, slots = case
     p, q = KEYS[name]
     pub, priv = flb.key_from_primes(p, q)
-    if slots == 0:
-        slots = pub.slot_capacity(qb + pb)
-        if slots == 0:
-            pytest.skip("toy key too small for this slot width")
     cd = flb.Codec(alpha, qb, pb, slots)
     n = 5 * slots + 3  # ragged tail
     x = _values(n, 7)

@@ -175,7 +175,7 @@ def test_tc_multi_tile_per_cta_both_problems():
 
 
 @pytest.mark.parametrize("words", [32, 64])
-@pytest.mark.parametrize("square", [False, True])
+@pytest.mark.parametrize("square", [0, 1, 2], ids=["general", "sqr_tri", "sqr_split"])
 def test_tc_product_phase_exact(words, square):
     """The tensor-core kernel's CUDA-core product phase (general row scan, or the block squaring
     of a^2) gives the exact 2w-limb integer product on random and extreme operands."""
@@ -193,11 +193,14 @@ def test_tc_product_phase_exact(words, square):
 
 
 @pytest.mark.parametrize("words", [32, 64])
-def test_tc_square_block_carries(words):
+@pytest.mark.parametrize("sq", [1, 2], ids=["tri", "split"])
+def test_tc_square_block_carries(words, sq):
     """Block squaring with triangular diagonal blocks (sqr_local: sum_{i<j} a_i a_j by lo/hi row
     chains, doubled, plus a_i^2): operands whose 16-limb lane blocks are all-ones, zero, or
     alternate 0xffffffff / 1 limbs, so every row chain, the doubling's shifted-out bits and the
-    quarter carries hit their extremes; exact 2w-limb a^2."""
+    quarter carries hit their extremes; exact 2w-limb a^2.  sq = 2: the half-split diagonal square
+    (two X/2 triangles + the doubled L H block rippled to the top), the form decryption and stage 1
+    of the key-holder encryption use."""
     X, nb = 16, words // 16
     full = (1 << (32 * X)) - 1
     alt = sum((0xFFFFFFFF if j % 2 == 0 else 1) << (32 * j) for j in range(X))
@@ -208,9 +211,12 @@ def test_tc_square_block_carries(words):
             vals.append(blk << (32 * X * kb))                                  # one block set
         vals.append(sum(blk << (32 * X * kb) for kb in range(nb)))             # every block
         vals.append(sum(blk << (32 * X * kb) for kb in range(0, nb, 2)))       # alternate blocks
+    half = (1 << (32 * X // 2)) - 1
+    for blk in (half, half << (32 * X // 2), (half << (32 * X // 2)) | 1):  # L or H half all-ones
+        vals.append(sum(blk << (32 * X * kb) for kb in range(nb)))
     vals += synthetic.uniform_below(1 << (32 * words), 128 - len(vals), 7150 + words)
     a = to_dev(vals, words)
-    t = from_dev(flb.debug_tc_product(a, a, square=True))
+    t = from_dev(flb.debug_tc_product(a, a, square=sq))
     for i, v in enumerate(vals):
         assert t[i] == v * v, (i, hex(t[i] ^ (v * v)))
 
