@@ -212,6 +212,43 @@ int flb_mod_pow_shared(const flb_mod* mod, const uint32_t* base, const uint32_t*
 int flb_rsa_keygen(uint32_t key_bits, uint64_t seed, uint32_t e, uint32_t* n_out, uint32_t* d_out,
                    uint32_t* p_out, uint32_t* q_out);
 
+/* ---------------------------------------------------------------- Table I fundamentals (NEXT-4)
+ * PAPER Table I (L241–L244) and §IV-D (L269–L273): "add/sub/mul/div ... compute the addition,
+ * subtraction, multiplication, and division of two multi-precision integer arrays", "mod computes
+ * the remainder", "mod_inv computes the modular inverse ... used to generate key pair[s]".
+ * Element-wise over batches of UNSIGNED integers: every operand is a device array
+ * [count][words] of little-endian u32 limbs, 1 <= words <= 256 (any width; rows 16-byte aligned
+ * when words % 4 == 0, else read limb by limb).  Each element runs on a group of lanes in the
+ * smallest frame of 32/64/128/256 limbs >= words (csrc/flb_mp.cu).  Asynchronous on `stream`.
+ * Errors: FLB_EINVAL (null pointer, words outside [1, 256]), FLB_ECUDA. */
+
+/* out_i = (a_i + b_i) mod 2^(32 words); carry (optional, uint32 [count]) = the carry out (0/1). */
+int flb_mp_add(const uint32_t* a, const uint32_t* b, uint32_t* out, uint32_t* carry, uint32_t words,
+               size_t count, void* stream);
+
+/* out_i = (a_i - b_i) mod 2^(32 words); borrow (optional) = 1 iff a_i < b_i. */
+int flb_mp_sub(const uint32_t* a, const uint32_t* b, uint32_t* out, uint32_t* borrow, uint32_t words,
+               size_t count, void* stream);
+
+/* out_i = a_i b_i, the full product: out is [count][2 words]. */
+int flb_mp_mul(const uint32_t* a, const uint32_t* b, uint32_t* out, uint32_t words, size_t count,
+               void* stream);
+
+/* q_i = floor(a_i / b_i), r_i = a_i mod b_i (either output may be NULL, not both); b_i = 0 gives
+ * q_i = 2^(32 words) - 1 and r_i = a_i (binary restoring division with a zero divisor). */
+int flb_mp_divmod(const uint32_t* a, const uint32_t* b, uint32_t* q, uint32_t* r, uint32_t words,
+                  size_t count, void* stream);
+
+/* Table I mod(x, n): r_i = x_i mod n_i (flb_mp_divmod's remainder; n_i = 0 gives x_i). */
+int flb_mp_mod(const uint32_t* x, const uint32_t* n, uint32_t* r, uint32_t words, size_t count,
+               void* stream);
+
+/* Table I mod_inv(x, n): out_i = x_i^-1 mod n_i in [1, n_i) when n_i >= 2 and gcd(x_i, n_i) = 1
+ * (any n_i, odd or even, e.g. d = e^-1 mod phi(n) for RSA); otherwise out_i = 0.  ok (optional,
+ * uint32 [count]) = 1 iff the inverse exists. */
+int flb_mp_mod_inv(const uint32_t* x, const uint32_t* n, uint32_t* out, uint32_t* ok, uint32_t words,
+                   size_t count, void* stream);
+
 /* ---------------------------------------------------------------- GPU key generation (NEXT-3)
  * "random number generator for large integers (including Miller-Rabin large prime
  * number generator)".  flb_miller_rabin runs `rounds` Miller–Rabin rounds on a batch of odd

@@ -23,7 +23,8 @@ __all__ = [
     "PublicKey", "PrivateKey", "keygen", "key_from_primes", "encrypt", "encrypt_crt", "decrypt", "add",
     "scalar_mul", "reduce_segments", "multiexp_segments", "pack", "unpack", "unpack_sums", "debug_mont_mul",
     "Codec", "FlbError", "library_path", "op_cost", "keygen_gpu", "miller_rabin", "Modulus", "rsa_keygen", "pack_encrypt_host", "decrypt_unpack_host",
-    "reduce_segments_host", "pack_encrypt_host_multi",
+    "reduce_segments_host", "pack_encrypt_host_multi", "mp_add", "mp_sub", "mp_mul", "mp_divmod", "mp_mod",
+    "mp_mod_inv",
 ]
 
 library_path = _lib.LIB_PATH
@@ -412,6 +413,87 @@ def rsa_keygen(key_bits: int, seed: int, e: int = 65537) -> Tuple[int, int, int,
     check("flb_rsa_keygen", LIB.flb_rsa_keygen(key_bits, seed & 0xFFFFFFFFFFFFFFFF, e, n, d, p, q))
     to_int = lambda a: sum(int(x) << (32 * i) for i, x in enumerate(a))
     return to_int(n), e, to_int(d), to_int(p), to_int(q)
+
+
+# ----------------------------------------------------------------------------- Table I fundamentals
+def _mp_operands(a: torch.Tensor, b: torch.Tensor, name_a: str = "a", name_b: str = "b") -> Tuple[int, int]:
+    if a.dim() != 2:
+        raise ValueError("%s must be [count, words]" % name_a)
+    words = a.shape[1]
+    M = _check_batch(a, words, name_a)
+    _check_batch(b, words, name_b, rows=M, like=a)
+    return M, words
+
+
+def _mp_flag(flag, M, like):
+    if flag is None:
+        return None
+    _check_vec(flag, (torch.int32, torch.uint32), "flag", M, like)
+    return flag
+
+
+def mp_add(a: torch.Tensor, b: torch.Tensor, out=None, carry=None, stream=None) -> torch.Tensor:
+    """Table I add: (a + b) mod 2^(32 words) per row; ``carry`` (int32 [count]) receives the
+    carry out."""
+    M, w = _mp_operands(a, b)
+    out = torch.empty_like(a) if out is None else out
+    _check_batch(out, w, "out", rows=M, like=a)
+    with _on(a):
+        check("flb_mp_add", LIB.flb_mp_add(_ptr(a), _ptr(b), _ptr(out), _ptr(_mp_flag(carry, M, a)), w, M,
+                                           _stream(stream)))
+    return out
+
+
+def mp_sub(a: torch.Tensor, b: torch.Tensor, out=None, borrow=None, stream=None) -> torch.Tensor:
+    """Table I sub: (a - b) mod 2^(32 words); ``borrow`` = 1 where a < b."""
+    M, w = _mp_operands(a, b)
+    out = torch.empty_like(a) if out is None else out
+    _check_batch(out, w, "out", rows=M, like=a)
+    with _on(a):
+        check("flb_mp_sub", LIB.flb_mp_sub(_ptr(a), _ptr(b), _ptr(out), _ptr(_mp_flag(borrow, M, a)), w, M,
+                                           _stream(stream)))
+    return out
+
+
+def mp_mul(a: torch.Tensor, b: torch.Tensor, out=None, stream=None) -> torch.Tensor:
+    """Table I mul: the full product a b, [count, 2 words]."""
+    M, w = _mp_operands(a, b)
+    out = torch.empty((M, 2 * w), dtype=torch.int32, device=a.device) if out is None else out
+    _check_batch(out, 2 * w, "out", rows=M, like=a)
+    with _on(a):
+        check("flb_mp_mul", LIB.flb_mp_mul(_ptr(a), _ptr(b), _ptr(out), w, M, _stream(stream)))
+    return out
+
+
+def mp_divmod(a: torch.Tensor, b: torch.Tensor, stream=None) -> Tuple[torch.Tensor, torch.Tensor]:
+    """Table I div and mod (L243): (floor(a / b), a mod b); b = 0 gives (2^(32 words) - 1, a)."""
+    M, w = _mp_operands(a, b)
+    q, r = torch.empty_like(a), torch.empty_like(a)
+    with _on(a):
+        check("flb_mp_divmod", LIB.flb_mp_divmod(_ptr(a), _ptr(b), _ptr(q), _ptr(r), w, M, _stream(stream)))
+    return q, r
+
+
+def mp_mod(x: torch.Tensor, n: torch.Tensor, out=None, stream=None) -> torch.Tensor:
+    """Table I mod(x, n): x mod n per row."""
+    M, w = _mp_operands(x, n, "x", "n")
+    out = torch.empty_like(x) if out is None else out
+    _check_batch(out, w, "out", rows=M, like=x)
+    with _on(x):
+        check("flb_mp_mod", LIB.flb_mp_mod(_ptr(x), _ptr(n), _ptr(out), w, M, _stream(stream)))
+    return out
+
+
+def mp_mod_inv(x: torch.Tensor, n: torch.Tensor, out=None, ok=None, stream=None) -> torch.Tensor:
+    """Table I mod_inv(x, n): x^-1 mod n per row (any n >= 2); 0 where no inverse exists
+    (``ok`` = 0 there)."""
+    M, w = _mp_operands(x, n, "x", "n")
+    out = torch.empty_like(x) if out is None else out
+    _check_batch(out, w, "out", rows=M, like=x)
+    with _on(x):
+        check("flb_mp_mod_inv", LIB.flb_mp_mod_inv(_ptr(x), _ptr(n), _ptr(out), _ptr(_mp_flag(ok, M, x)), w, M,
+                                                   _stream(stream)))
+    return out
 
 
 # ----------------------------------------------------------------------------- host-buffer pipeline

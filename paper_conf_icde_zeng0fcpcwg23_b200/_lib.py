@@ -63,6 +63,12 @@ SIGNATURES = {
     "flb_mod_pow": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),
     "flb_mod_pow_shared": (ctypes.c_int, [_P, _P, _P, _U32, _P, _SZ, _P]),
     "flb_rsa_keygen": (ctypes.c_int, [_U32, _U64, _U32, _P, _P, _P, _P]),
+    "flb_mp_add": (ctypes.c_int, [_P, _P, _P, _P, _U32, _SZ, _P]),
+    "flb_mp_sub": (ctypes.c_int, [_P, _P, _P, _P, _U32, _SZ, _P]),
+    "flb_mp_mul": (ctypes.c_int, [_P, _P, _P, _U32, _SZ, _P]),
+    "flb_mp_divmod": (ctypes.c_int, [_P, _P, _P, _P, _U32, _SZ, _P]),
+    "flb_mp_mod": (ctypes.c_int, [_P, _P, _P, _U32, _SZ, _P]),
+    "flb_mp_mod_inv": (ctypes.c_int, [_P, _P, _P, _P, _U32, _SZ, _P]),
     "flb_miller_rabin": (ctypes.c_int, [_P, _U32, _P, _U32, _U64, _P, _SZ, _P]),
     "flb_keygen_gpu": (ctypes.c_int, [_U32, _U64, ctypes.POINTER(_P), ctypes.POINTER(_P), _P]),
     "flb_pack_encrypt_host": (ctypes.c_int, [_P, _P, ctypes.POINTER(CodecStruct), _P, _SZ, _U64, _U64, _P]),

@@ -360,17 +360,7 @@ __device__ __forceinline__ void mul_full(uint32_t (&lo)[X], uint32_t (&hi)[X], c
   collapse<X, T>(hi, E, O, pend);
 }
 
-// ----------------------------------------------------------------------------- squaring
-// Montgomery squaring with the square computed by lane-local X x X block products (PAPER L207:
-// squarings are ~87 % of a modexp's multiplications).  a^2 = sum_k A_k^2 2^(2 k X w) +
-// 2 sum_{k<l} A_k A_l 2^((k+l) X w), A_k = lane k's chunk.  Lane k computes its square block and
-// the cross blocks (k, k+d mod T) for d = 1 .. T/2-1, plus d = T/2 when k < T/2 — every
-// unordered pair exactly once, T/2 + 1 blocks per lane (vs T rows of CIOS products): 1280 instead
-// of 2048 limb products per lane at T = 8.  Blocks are summed (cross blocks doubled) into 64-bit
-// column sums in shared memory — two non-overlapping write phases per block round, no atomics —
-// then one carry normalisation gives t = a^2 as (t_lo, t_hi) in the CIOS layout, and a reduce-only
-// CIOS pass gives REDC(t_lo) + t_hi = a^2 R^-1 (mod N), < 2N, canonicalised.
-
+// ----------------------------------------------------------------------------- lane-local rows
 // lane-local product row: acc += a * bi (no neighbour lanes), shift one word, return the word out
 template <int X>
 __device__ __forceinline__ uint32_t local_row(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
@@ -389,108 +379,6 @@ __device__ __forceinline__ uint32_t local_row(uint32_t (&E)[X + 1], uint32_t (&O
   nO[X] = 0;
 #pragma unroll
   for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
-  return out;
-}
-
-// per-group 64-bit column sums for the 2S-word square
-template <int X, int T>
-__device__ __forceinline__ unsigned long long* col_group() {
-  constexpr int S = X * T;
-  __shared__ __align__(16) unsigned long long cbuf[kMaxWarps * 32 / T * 2 * S];
-  return cbuf + ((threadIdx.x >> 5) * (32 / T) + (int)((lane_id() & 31u) / T)) * (2 * S);
-}
-
-// reduce-only CIOS step: m = word0 * n0inv; acc += m N; acc >>= 32
-template <int X, int T>
-__device__ __forceinline__ void redc_step(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
-                                          const uint32_t (&n)[X], uint32_t n0inv) {
-  const int k = (int)(lane_id() & (T - 1));
-  // merge the pending word into word 0; its carry enters the O chain (word 1) after m is formed
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
-  const uint32_t m = __shfl_sync(FULL, E[0], 0, T) * n0inv;
-  chain_odd<X, true>(O, n, m);
-  chain_even<X>(E, n, m);
-  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
-  if (k == T - 1) up = 0;
-  pend = E[1];
-  uint32_t nE[X + 1], nO[X + 1];
-#pragma unroll
-  for (int t = 0; t <= X; t++) nE[t] = O[t];
-#pragma unroll
-  for (int t = 0; t + 2 <= X; t++) nO[t] = E[t + 2];
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[X - 2]) : "r"(up));
-  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[X - 1]));
-  nO[X] = 0;
-#pragma unroll
-  for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
-}
-
-// ----------------------------------------------------------------------------- split squaring
-// Montgomery squaring with a quarter of the square's limb products moved out of the reduced part.
-// With B = 2^(32 S/2), R = B^2 and a = L + H B (L, H the low / high halves of a):
-//   a^2 = t_A + H^2 R,   t_A = L^2 + 2 L H B = L (L + 2 H B),
-// so a^2 R^-1 = (t_A + m N) / R + H^2 (mod N) for the m that REDC(t_A) picks: H^2 R is an exact
-// multiple of R and needs no reduction.  The reduced part is a CIOS over the S/2 multiplier words of
-// L against a'' = L + 2 H B (phase 1, S/2 full steps) followed by S/2 reduce-only steps (phase 2);
-// the plain half-size square H^2 is spread over all T lanes (X/2 words each) and its rows are
-// interleaved with phase 2, whose m-broadcast latency they hide.  Limb products: S^2/2 + S^2 + S^2/4
-// = 1.75 S^2 instead of CIOS's 2 S^2.  Bound: (t_A + m N)/R + H^2 = (a^2 + m N)/R < 2N for a < N, so
-// one conditional subtraction canonicalises, as for mont_mul.
-//
-// Phase-1 step: cios_step<REDUCE> plus `top` added at word X of the lane (word S of the group for
-// lane T-1: the product of b_i with the 2H top bit).
-template <int X, int T>
-__device__ __forceinline__ void cios_step_top(uint32_t (&E)[X + 1], uint32_t (&O)[X + 1], uint32_t& pend,
-                                              const uint32_t (&a)[X], uint32_t bi, uint32_t top,
-                                              const uint32_t (&n)[X], uint32_t n0inv) {
-  const int k = (int)(lane_id() & (T - 1));
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
-  chain_odd<X, true>(O, a, bi);
-  chain_even<X>(E, a, bi);
-  const uint32_t m = __shfl_sync(FULL, E[0], 0, T) * n0inv;
-  chain_even<X>(E, n, m);
-  chain_odd<X, false>(O, n, m);
-  // after both chains (their closing addc into E[X] / O[X] assume small top words); the shift
-  // below moves E[X] into a regular chain word, so a large value there is safe
-  asm volatile("add.cc.u32 %0, %0, %2;\n\taddc.u32 %1, %1, 0;" : "+r"(E[X]), "+r"(O[X]) : "r"(top));
-  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
-  if (k == T - 1) up = 0;
-  pend = E[1];
-  uint32_t nE[X + 1], nO[X + 1];
-#pragma unroll
-  for (int t = 0; t <= X; t++) nE[t] = O[t];
-#pragma unroll
-  for (int t = 0; t + 2 <= X; t++) nO[t] = E[t + 2];
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[X - 2]) : "r"(up));
-  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[X - 1]));
-  nO[X] = 0;
-#pragma unroll
-  for (int t = 0; t <= X; t++) { E[t] = nE[t]; O[t] = nO[t]; }
-}
-
-// Plain product row over HX words per lane (no reduction): acc += a * bi, shift one word down the
-// group.  Returns lane 0's word shifted out (the product's next low word; meaningful in lane 0).
-template <int HX, int T>
-__device__ __forceinline__ uint32_t prod_step(uint32_t (&E)[HX + 1], uint32_t (&O)[HX + 1], uint32_t& pend,
-                                              const uint32_t (&a)[HX], uint32_t bi) {
-  const int k = (int)(lane_id() & (T - 1));
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(E[0]) : "r"(pend));
-  chain_odd<HX, true>(O, a, bi);
-  chain_even<HX>(E, a, bi);
-  const uint32_t out = E[0];
-  uint32_t up = __shfl_down_sync(FULL, E[0], 1, T);
-  if (k == T - 1) up = 0;
-  pend = E[1];
-  uint32_t nE[HX + 1], nO[HX + 1];
-#pragma unroll
-  for (int t = 0; t <= HX; t++) nE[t] = O[t];
-#pragma unroll
-  for (int t = 0; t + 2 <= HX; t++) nO[t] = E[t + 2];
-  asm volatile("add.cc.u32 %0, %0, %1;" : "+r"(nO[HX - 2]) : "r"(up));
-  asm volatile("addc.u32 %0, 0, 0;" : "=r"(nO[HX - 1]));
-  nO[HX] = 0;
-#pragma unroll
-  for (int t = 0; t <= HX; t++) { E[t] = nE[t]; O[t] = nO[t]; }
   return out;
 }
 
