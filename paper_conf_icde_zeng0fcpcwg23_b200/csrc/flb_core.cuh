@@ -566,7 +566,13 @@ int launch_tc_exp_dag(flb::tc::ExpArgs& A1, flb::tc::ExpArgs& A2, cudaStream_t s
     return fail(FLB_EINVAL, "dag launch: the two stages must have the same problems' tile counts");
   if (t1 == 0) return FLB_OK;
   if (t1 >= 0xFFFFFFF0ull / 2) return fail(FLB_EINVAL, "dag launch: too many tiles");
-  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), t1 + t2);
+  // CTAs per SM (2: one tile's product phase overlaps the other's MMA / normalisation); FLB_TC_CPS=1
+  // is a measurement knob (one tile per SM, no overlap)
+  static const int cps = [] {
+    const char* e = getenv("FLB_TC_CPS");
+    return (e && atoi(e) == 1) ? 1 : 2;
+  }();
+  const int grid = (int)std::min<uint64_t>((uint64_t)(cps * sms), t1 + t2);
   const uint64_t stride = (uint64_t)flb::tc::kTileM * std::max<uint64_t>((uint64_t)(tab1 + 1) * S1,
                                                                           (uint64_t)(tab2 + 1) * S2);
   Scratch s_tab, s_sync;

@@ -21,12 +21,12 @@ FLB_TC_DAG_DECLS()
 #if defined(FLB_INST_TC) && FLB_INST_TC == 64 && FLB_TC_PROF
 // profiling builds only (FLB_NVCC_EXTRA=-DFLB_TC_PROF=1; not in include/): per-phase cycle totals of
 // thread 0 of the 2048-bit tensor-core Montgomery kernel (tools/tc_phases.py)
-extern "C" int flb_debug_tc_prof(uint64_t* out8, int reset) {
-  unsigned long long h[8];
+extern "C" int flb_debug_tc_prof(uint64_t* out16, int reset) {
+  unsigned long long h[16];
   FLB_CK(cudaMemcpyFromSymbol(h, flb::tc::g_tc_prof, sizeof(h)));
-  for (int i = 0; i < 8; i++) out8[i] = h[i];
+  for (int i = 0; i < 16; i++) out16[i] = h[i];
   if (reset) {
-    unsigned long long z[8] = {};
+    unsigned long long z[16] = {};
     FLB_CK(cudaMemcpyToSymbol(flb::tc::g_tc_prof, z, sizeof(z)));
   }
   return FLB_OK;

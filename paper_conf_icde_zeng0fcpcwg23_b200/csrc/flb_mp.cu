@@ -281,7 +281,9 @@ __global__ void __launch_bounds__(32) k_mp_modinv(const MpArgs A) {
     uint32_t one[X], d[X];
     zero_limbs<X>(one);
     if (k == 0) one[0] = 1;
-    const bool n_big = grp_sub<X, T>(d, n, one) == 0u && !grp_is_zero<T>(d);
+    const uint32_t nb = grp_sub<X, T>(d, n, one);  // (both collectives run in every group: no short circuit)
+    const bool n1 = grp_is_zero<T>(d);
+    const bool n_big = nb == 0u && !n1;
     // odd n: (u0, M) = (x mod n, n); even n: (n mod x, x)
     uint32_t A0[X], M[X], u0[X];
     sel(A0, n_odd, x, n);

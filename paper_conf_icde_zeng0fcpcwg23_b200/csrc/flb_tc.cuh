@@ -151,11 +151,6 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t* v) {
 }
 __device__ __forceinline__ void tmem_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
-// four byte-column sums (each < 2^25) as one 32-bit-word contribution
-__device__ __forceinline__ uint64_t word_of(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3) {
-  return (uint64_t)c0 + ((uint64_t)c1 << 8) + ((uint64_t)c2 << 16) + ((uint64_t)c3 << 24);
-}
-
 // carry-flag chains (one IADD3(.X) per word; the flag lives between consecutive asm statements,
 // which no other instruction of this file touches)
 __device__ __forceinline__ uint32_t add_cc(uint32_t a, uint32_t b) {
@@ -189,25 +184,47 @@ __device__ __forceinline__ uint32_t subc_end(uint32_t a, uint32_t b) {
   return r;
 }
 
-// Normalise 8 words of byte-column sums (plus optional addends th) into v[0..8): with the 64-bit
-// word values W_w = word_of(cols 4w..4w+3) (+ th[w]), off the chain, the sum is
-// sum_w (lo W_w + hi W_(w-1)) 2^(32w), one addc.cc per word; `hprev` carries hi W of the last word
-// into the next chunk (the flag carries the rest).  first: the chain starts here (add.cc).
+// Normalise 8 words of byte-column sums c_j (each < 2^25; j = 4w + r) plus optional addends th_w
+// into v[0..8), entirely on the integer ALU pipe (the FMA-heavy pipe carries the limb products).
+// sum_j c_j 2^(8j) = C_0 + 2^8 C_1 + 2^16 C_2 + 2^24 C_3 with C_r = sum_w c_(4w+r) 2^(32w): word w of
+// 2^(8r) C_r is the funnel shift of c_(4w+r) with the previous word's c_(4w-4+r) (its bits above
+// 2^32 spill into word w + 1), so word w of the sum is the 64-bit S_w = c_4w + f1_w + f2_w + f3_w
+// (+ th_w) (IADD3 pairs, off the carry chain) and v_w = lo S_w + hi S_(w-1) + flag (one addc.cc
+// per word).  State across chunks: the last columns of residues 1..3 (p1..p3) and hi S of the last
+// word (hprev).  first: the chain starts here (add.cc).
+struct NormState {
+  uint32_t p1 = 0, p2 = 0, p3 = 0, hprev = 0;
+  // everything above the normalised words: the final flag + hi S of the last word + the spills of
+  // the last word's shifted columns
+  __device__ __forceinline__ uint32_t carry_out_end() {
+    return addc_end(hprev, 0u) + (p1 >> 24) + (p2 >> 16) + (p3 >> 8);
+  }
+};
 template <bool TH>
-__device__ __forceinline__ void norm8_chain(const uint32_t (&cv)[32], const uint32_t* th, uint32_t* v,
-                                            uint32_t& hprev, bool first) {
+__device__ __forceinline__ void norm8_chain(const uint32_t (&cv)[32], const uint32_t* th, uint32_t* v, NormState& st,
+                                            bool first) {
   uint32_t lo[8], hi[8];
+  uint32_t p1 = st.p1, p2 = st.p2, p3 = st.p3;
 #pragma unroll
   for (int w = 0; w < 8; w++) {
-    uint64_t W = word_of(cv[4 * w], cv[4 * w + 1], cv[4 * w + 2], cv[4 * w + 3]);
-    if (TH) W += th[w];
-    lo[w] = (uint32_t)W;
-    hi[w] = (uint32_t)(W >> 32);
+    const uint32_t f1 = __funnelshift_l(p1, cv[4 * w + 1], 8);
+    const uint32_t f2 = __funnelshift_l(p2, cv[4 * w + 2], 16);
+    const uint32_t f3 = __funnelshift_l(p3, cv[4 * w + 3], 24);
+    p1 = cv[4 * w + 1];
+    p2 = cv[4 * w + 2];
+    p3 = cv[4 * w + 3];
+    uint64_t S = (uint64_t)cv[4 * w] + f1 + f2;
+    S += TH ? (uint64_t)f3 + th[w] : (uint64_t)f3;
+    lo[w] = (uint32_t)S;
+    hi[w] = (uint32_t)(S >> 32);
   }
-  v[0] = first ? add_cc(lo[0], hprev) : addc_cc(lo[0], hprev);
+  st.p1 = p1;
+  st.p2 = p2;
+  st.p3 = p3;
+  v[0] = first ? add_cc(lo[0], st.hprev) : addc_cc(lo[0], st.hprev);
 #pragma unroll
   for (int w = 1; w < 8; w++) v[w] = addc_cc(lo[w], hi[w - 1]);
-  hprev = hi[7];
+  st.hprev = hi[7];
 }
 
 struct Smem {
@@ -263,15 +280,16 @@ __device__ __forceinline__ uint32_t ld_u32(const uint32_t* p, uint32_t ld) {
 #define FLB_TC_PROF 0
 #endif
 #if FLB_TC_PROF
-// per-phase cycle totals of thread 0 (P, M1 wait, N1, M2 wait, F, calls): FLB_TC_PROF=1 builds only
-static __device__ unsigned long long g_tc_prof[8];
-#define TC_MARK(slot)                                               \
-  do {                                                              \
-    if (threadIdx.x == 0) {                                         \
-      const long long now_ = clock64();                             \
-      atomicAdd(&g_tc_prof[slot], (unsigned long long)(now_ - t_)); \
-      t_ = now_;                                                    \
-    }                                                               \
+// per-phase cycle totals of thread 0 (P, M1 wait, N1, M2 wait, F, calls), slots [0, 8) for S = 32
+// and [8, 16) for S = 64: FLB_TC_PROF=1 builds only
+static __device__ unsigned long long g_tc_prof[16];
+#define TC_MARK(slot)                                                                   \
+  do {                                                                                  \
+    if (threadIdx.x == 0) {                                                             \
+      const long long now_ = clock64();                                                 \
+      atomicAdd(&g_tc_prof[(S == 64 ? 8 : 0) + (slot)], (unsigned long long)(now_ - t_)); \
+      t_ = now_;                                                                        \
+    }                                                                                   \
   } while (0)
 #else
 #define TC_MARK(slot) do {} while (0)
@@ -348,10 +366,35 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 
 // v = a^2 (2X words) for this lane's own block, X (X - 1) / 2 + X limb products instead of X^2
 // (squarings dominate the modexp).  U = sum_{i<j} a_i a_j 2^(32 (i + j)) by rows
-// j = 0 .. X - 2 (row j: a[j+1, X) x a_j at word 2j + 1, a lo chain then a hi chain one word up),
-// then v = 2 U + sum_i a_i^2 2^(64 i) in one carry chain with the doubling as a funnel shift.
-// Bounds: after row j the partial sum is < 2^(32 (X + j + 1)), so neither chain carries past word
-// X + j + 1; 2 U + D = a^2 < 2^(64 X), so the final chain has no carry out.
+// j = 0 .. X - 2 (row j: a[j+1, X) x a_j from word 2j + 1), then v = 2 U + sum_i a_i^2 2^(64 i) in
+// one carry chain with the doubling as a funnel shift.  Each product's (lo, hi) goes to the aligned
+// word pair (i + j, i + j + 1), so a row is two carry chains of whole products — i = j+1, j+3, ..
+// (odd pairs) and i = j+2, j+4, .. (even pairs) — and every product is one IMAD.WIDE.U32(.X)
+// (ptxas fuses the mad.lo.cc / madc.hi.cc pair), not a separate IMAD + IMAD.HI.
+// Bounds: U plus any subset of row j's products is < 2^(32 (X + j + 1)), so a chain that ends at
+// word X + j drops its carry and one that ends at X + j - 1 carries into word X + j only.
+template <int X>
+__device__ __forceinline__ void sqr_row_chain(uint32_t (&u)[2 * X], const uint32_t (&a)[X], int j, int i0) {
+#pragma unroll
+  for (int i = i0; i < X; i += 2) {
+    const int p = i + j;
+    const bool first = i == i0, last = i + 2 >= X;
+    if (first && last && p + 1 == X + j)
+      asm volatile("mad.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.u32 %1, %2, %3, %1;"
+                   : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
+    else if (first)
+      asm volatile("mad.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.cc.u32 %1, %2, %3, %1;"
+                   : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
+    else if (last && p + 1 == X + j)
+      asm volatile("madc.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.u32 %1, %2, %3, %1;"
+                   : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
+    else
+      asm volatile("madc.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.cc.u32 %1, %2, %3, %1;"
+                   : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
+    if (last && p + 1 == X + j - 1) asm volatile("addc.u32 %0, %0, 0;" : "+r"(u[X + j]));
+  }
+}
+
 template <int X>
 __device__ __forceinline__ void sqr_local(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
   uint32_t u[2 * X];
@@ -359,24 +402,8 @@ __device__ __forceinline__ void sqr_local(uint32_t (&v)[2 * X], const uint32_t (
   for (int w = 0; w < 2 * X; w++) u[w] = 0;
 #pragma unroll
   for (int j = 0; j < X - 1; j++) {
-    // lo chain: u[i + j] += lo(a_i a_j), i = j+1 .. X-1; carry into u[X + j] (<= 1 before: no carry out)
-#pragma unroll
-    for (int i = j + 1; i < X; i++) {
-      if (i == j + 1)
-        asm volatile("mad.lo.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j]) : "r"(a[i]), "r"(a[j]));
-      else
-        asm volatile("madc.lo.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j]) : "r"(a[i]), "r"(a[j]));
-    }
-    asm volatile("addc.u32 %0, %0, 0;" : "+r"(u[X + j]));
-    // hi chain: u[i + j + 1] += hi(a_i a_j); carry into the fresh word u[X + j + 1]
-#pragma unroll
-    for (int i = j + 1; i < X; i++) {
-      if (i == j + 1)
-        asm volatile("mad.hi.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j + 1]) : "r"(a[i]), "r"(a[j]));
-      else
-        asm volatile("madc.hi.cc.u32 %0, %1, %2, %0;" : "+r"(u[i + j + 1]) : "r"(a[i]), "r"(a[j]));
-    }
-    asm volatile("addc.u32 %0, 0, 0;" : "=r"(u[X + j + 1]));
+    sqr_row_chain<X>(u, a, j, j + 1);
+    if (j + 2 < X) sqr_row_chain<X>(u, a, j, j + 2);
   }
   // v = 2 U + D
 #pragma unroll
@@ -726,15 +753,15 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   };
   // ---- N1: q = D1 mod R
   {
-    uint32_t hprev = 0;
+    NormState ns;
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
       uint32_t cv[32];
       tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
       tmem_wait();
-      norm8_chain<false>(cv, nullptr, v + c0 / 4, hprev, c0 == 0);
+      norm8_chain<false>(cv, nullptr, v + c0 / 4, ns, c0 == 0);
     }
-    publish(addc_end(hprev, 0u));
+    publish(ns.carry_out_end());
   }
   tc_before_sync();
   __syncthreads();  // D1 drained, t_lo bytes read, carries published
@@ -765,11 +792,15 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       uint32_t bc[8];
       tmem_ld8(lane_base, bc);
       tmem_wait();
-      const uint64_t s0 = word_of(bc[0], bc[1], bc[2], bc[3]) + ttop.x;
-      const uint64_t s1 = (s0 >> 32) + word_of(bc[4], bc[5], bc[6], bc[7]) + ttop.y;
-      carry = (s1 >> 32) + ((((uint32_t)s0) | ((uint32_t)s1)) != 0u ? 1u : 0u);
+      // W as two words (the funnel-shift form of norm8_chain, on the ALU pipe)
+      const uint64_t s0 = (uint64_t)bc[0] + (bc[1] << 8) + (bc[2] << 16) + (uint64_t)(bc[3] << 24) + ttop.x;
+      const uint64_t s1 = (s0 >> 32) + bc[4] + __funnelshift_l(bc[1], bc[5], 8) + __funnelshift_l(bc[2], bc[6], 16) +
+                          (uint64_t)__funnelshift_l(bc[3], bc[7], 24) + ttop.y;
+      const uint64_t top = (s1 >> 32) + (bc[5] >> 24) + (bc[6] >> 16) + (bc[7] >> 8);
+      carry = top + ((((uint32_t)s0) | ((uint32_t)s1)) != 0u ? 1u : 0u);
     }
-    uint32_t hprev = (uint32_t)carry;  // < 2^20
+    NormState ns;
+    ns.hprev = (uint32_t)carry;  // < 2^20
     // this half's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; half 1's last 8 columns
     // (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
     uint32_t top[8] = {0, 0, 0, 0, 0, 0, 0, 0};
@@ -811,9 +842,9 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       const uint4 h0 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[0];
       const uint4 h1 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[1];
       const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
-      norm8_chain<true>(cv, th, v + c0 / 4, hprev, c0 == 0);
+      norm8_chain<true>(cv, th, v + c0 / 4, ns, c0 == 0);
     }
-    publish(addc_end(hprev, 0u));
+    publish(ns.carry_out_end());
   }
   tc_before_sync();
   __syncthreads();
@@ -856,7 +887,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   __syncthreads();
   TC_MARK(4);
 #if FLB_TC_PROF
-  if (threadIdx.x == 0) atomicAdd(&g_tc_prof[5], 1ull);
+  if (threadIdx.x == 0) atomicAdd(&g_tc_prof[(S == 64 ? 8 : 0) + 5], 1ull);
 #endif
 }
 

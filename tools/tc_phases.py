@@ -15,16 +15,19 @@ pub, priv = flb.keygen(2048, 0xF1B0 + 2048)
 m = torch.randint(0, 2**31 - 1, (count, 64), dtype=torch.int32).cuda()
 fn = flb.LIB.flb_debug_tc_prof
 fn.argtypes = [ctypes.POINTER(ctypes.c_uint64), ctypes.c_int]
-buf = (ctypes.c_uint64 * 8)()
+buf = (ctypes.c_uint64 * 16)()
 flb.encrypt_crt(priv, m, seed=1)
 torch.cuda.synchronize()
 fn(buf, 1)
 flb.encrypt_crt(priv, m, seed=1)
 torch.cuda.synchronize()
 fn(buf, 0)
-calls = buf[5]
 names = ["P (product + sA/t_hi writes + barrier)", "M1 issue + wait", "N1 (q normalise + resolve + sA)",
          "M2 wait", "F (finish + borrow + writes)"]
-tot = sum(buf[i] for i in range(5))
-print(json.dumps({"calls": calls, "cycles_per_call": tot / max(calls, 1),
-                  "phases": {n: round(buf[i] / max(calls, 1)) for i, n in enumerate(names)}}, indent=1))
+out = {}
+for S, o in ((32, 0), (64, 8)):
+    calls = buf[o + 5]
+    tot = sum(buf[o + i] for i in range(5))
+    out["S=%d" % S] = {"calls": calls, "cycles_per_call": tot / max(calls, 1),
+                       "phases": {n: round(buf[o + i] / max(calls, 1)) for i, n in enumerate(names)}}
+print(json.dumps(out, indent=1))
