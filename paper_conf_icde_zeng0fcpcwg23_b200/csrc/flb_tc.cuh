@@ -360,6 +360,9 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 #ifndef FLB_TC_TRISQ_S1
 #define FLB_TC_TRISQ_S1 2  // stage-1 tiles (S = 32) of k_tc_exp_dag: the half-split form
 #endif
+#ifndef FLB_TC_TRISQ_S2
+#define FLB_TC_TRISQ_S2 1  // stage-2 tiles (S = 64) of k_tc_exp_dag
+#endif
 #ifndef FLB_TC_TRISQ_EXP
 #define FLB_TC_TRISQ_EXP 2  // k_tc_exp (decryption; two-launch key-holder stages): the half-split form
 #endif
@@ -367,44 +370,53 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 // v = a^2 (2X words) for this lane's own block, X (X - 1) / 2 + X limb products instead of X^2
 // (squarings dominate the modexp).  U = sum_{i<j} a_i a_j 2^(32 (i + j)) by rows
 // j = 0 .. X - 2 (row j: a[j+1, X) x a_j from word 2j + 1), then v = 2 U + sum_i a_i^2 2^(64 i) in
-// one carry chain with the doubling as a funnel shift.  Each product's (lo, hi) goes to the aligned
-// word pair (i + j, i + j + 1), so a row is two carry chains of whole products — i = j+1, j+3, ..
-// (odd pairs) and i = j+2, j+4, .. (even pairs) — and every product is one IMAD.WIDE.U32(.X)
-// (ptxas fuses the mad.lo.cc / madc.hi.cc pair), not a separate IMAD + IMAD.HI.
-// Bounds: U plus any subset of row j's products is < 2^(32 (X + j + 1)), so a chain that ends at
-// word X + j drops its carry and one that ends at X + j - 1 carries into word X + j only.
-template <int X>
+// one carry chain with the doubling as a funnel shift.  Every product is one IMAD.WIDE.U32(.X)
+// (ptxas fuses a mad.lo.cc / madc.hi.cc pair into it), whose 64-bit accumulator must be an
+// even-aligned register pair: products at even words i + j accumulate into UE (pairs at even
+// indices), those at odd words into UO shifted down one word (UO[q] is word q + 1, pairs again at
+// even indices), so a row is two carry chains of whole products — i = j+2, j+4, .. into UE and
+// i = j+1, j+3, .. into UO — with no register moves; U = UE + 2^32 UO at the end.
+// Bounds: UE or UO plus any subset of row j's products is < 2^(32 (X + j + 1)), so a chain that
+// ends at word X + j drops its carry and one that ends at X + j - 1 carries into word X + j only.
+template <int X, int OFF>
 __device__ __forceinline__ void sqr_row_chain(uint32_t (&u)[2 * X], const uint32_t (&a)[X], int j, int i0) {
 #pragma unroll
   for (int i = i0; i < X; i += 2) {
-    const int p = i + j;
+    const int p = i + j - OFF;  // accumulator index of the product's low word
     const bool first = i == i0, last = i + 2 >= X;
-    if (first && last && p + 1 == X + j)
+    const bool top = i + j + 1 == X + j;  // the chain's last word is X + j: no carry out
+    if (first && last && top)
       asm volatile("mad.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.u32 %1, %2, %3, %1;"
                    : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
     else if (first)
       asm volatile("mad.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.cc.u32 %1, %2, %3, %1;"
                    : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
-    else if (last && p + 1 == X + j)
+    else if (last && top)
       asm volatile("madc.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.u32 %1, %2, %3, %1;"
                    : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
     else
       asm volatile("madc.lo.cc.u32 %0, %2, %3, %0;\n\tmadc.hi.cc.u32 %1, %2, %3, %1;"
                    : "+r"(u[p]), "+r"(u[p + 1]) : "r"(a[i]), "r"(a[j]));
-    if (last && p + 1 == X + j - 1) asm volatile("addc.u32 %0, %0, 0;" : "+r"(u[X + j]));
+    if (last && !top) asm volatile("addc.u32 %0, %0, 0;" : "+r"(u[X + j - OFF]));
   }
 }
 
 template <int X>
 __device__ __forceinline__ void sqr_local(uint32_t (&v)[2 * X], const uint32_t (&a)[X]) {
-  uint32_t u[2 * X];
+  uint32_t ue[2 * X], uo[2 * X], u[2 * X];
 #pragma unroll
-  for (int w = 0; w < 2 * X; w++) u[w] = 0;
+  for (int w = 0; w < 2 * X; w++) { ue[w] = 0; uo[w] = 0; }
 #pragma unroll
   for (int j = 0; j < X - 1; j++) {
-    sqr_row_chain<X>(u, a, j, j + 1);
-    if (j + 2 < X) sqr_row_chain<X>(u, a, j, j + 2);
+    sqr_row_chain<X, 1>(uo, a, j, j + 1);
+    if (j + 2 < X) sqr_row_chain<X, 0>(ue, a, j, j + 2);
   }
+  // U = UE + 2^32 UO (< 2^(32 (2X - 1))): no carry out of the top word
+  u[0] = ue[0];
+  u[1] = add_cc(ue[1], uo[0]);
+#pragma unroll
+  for (int w = 2; w < 2 * X - 1; w++) u[w] = addc_cc(ue[w], uo[w - 1]);
+  u[2 * X - 1] = addc_end(ue[2 * X - 1], uo[2 * X - 2]);
   // v = 2 U + D
 #pragma unroll
   for (int i = 0; i < X; i++) {
@@ -1165,7 +1177,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, co
         }
       }
       __syncthreads();
-      tc_exp_tile<S2>(P, tile, A2.one, tab, sm, phase, kLdGPU);  // y: written by another CTA of this launch
+      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, sm, phase, kLdGPU);  // y: written by another CTA of this launch
     } else {
       tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm, phase);
     }

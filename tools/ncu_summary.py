@@ -28,6 +28,11 @@ KEYS = {
     "stall_short_scoreboard": "smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio",
     "stall_long_scoreboard": "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
     "local_load_inst": "smsp__sass_inst_executed_op_local_ld.sum",
+    "fmaheavy_pipe_pct_active": "sm__pipe_fmaheavy_cycles_active.avg.pct_of_peak_sustained_active",
+    "alu_inst_pct_active": "sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active",
+    "stall_barrier": "smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio",
+    "warps_active_per_scheduler": "smsp__warps_active.avg.per_cycle_active",
+    "dram_throughput_pct": "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
 }
 
 
