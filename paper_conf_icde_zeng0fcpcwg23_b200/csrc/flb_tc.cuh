@@ -324,6 +324,20 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
   }
 }
 
+// Element of the tile that thread tid works on in product pass h (and in the row ops): the warp pair
+// (L, L + 4) that normalises elements [32 L, 32 L + 32) in tc_mont also owns them here, so every
+// per-element hand-off between phases needs only a barrier over that pair (named barrier 1 + L, 64
+// threads); only the MMA issues, which read all 128 rows, need the whole CTA.
+template <int S>
+__device__ __forceinline__ int prod_elem(int h) {
+  constexpr int T = Cfg<S>::T;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  return 32 * (warp & 3) + h * (64 / T) + (warp >> 2) * (32 / T) + (tid & 31) / T;
+}
+__device__ __forceinline__ void pair_sync() {
+  asm volatile("bar.sync %0, 64;" :: "r"(1 + ((threadIdx.x >> 5) & 3)) : "memory");
+}
+
 // ----------------------------------------------------------------------------- squaring product
 // t = a^2 for the product phase when a = b (87 % of the multiplications of a modexp).  Lane k of the
 // element's group holds the limb block a_k = a[kX, kX+X) (X = S/4).  a^2 is the sum of block
@@ -655,7 +669,7 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
   // ---- P: t = a b, NP passes of EP elements (S = 64: two passes of 64; S = 32: one of 128)
 #pragma unroll 1
   for (int h = 0; h < C::NP; h++) {
-    const int elem = h * C::EP + tid / T;
+    const int elem = prod_elem<S>(h);
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
     if constexpr (T == 2) {
@@ -775,8 +789,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
     publish(ns.carry_out_end());
   }
-  tc_before_sync();
-  __syncthreads();  // D1 drained, t_lo bytes read, carries published
+  pair_sync();  // carries published (D1 drained before M2: the CTA barrier below)
   if (g == 1) add_in(carry_out(0, 0));
 #pragma unroll
   for (int c = 0; c < QW / 4; c++)
@@ -858,8 +871,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
     publish(ns.carry_out_end());
   }
-  tc_before_sync();
-  __syncthreads();
+  pair_sync();
   const uint64_t c1 = carry_out(0, 0);
   const uint64_t ovf = carry_out(1, c1);  // bit above S words (u < 2N < 2R)
   if (g == 1) add_in(c1);
@@ -881,7 +893,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     for (int w = 0; w < QW; w++) nzd |= d[w];
     xch[g].w = br | (nzd == 0u ? 2u : 0u);
   }
-  __syncthreads();
+  pair_sync();
   {
     const uint32_t f0 = xch[0].w, f1 = xch[1].w;
     const uint32_t b1 = f0 & 1u;                          // borrow into half 1
@@ -896,7 +908,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       reinterpret_cast<uint4*>(row + g * QW)[c] = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
   }
   tc_before_sync();
-  __syncthreads();
+  pair_sync();  // the pair's rows are final (the next product / row op of these elements is the pair's)
   TC_MARK(4);
 #if FLB_TC_PROF
   if (threadIdx.x == 0) atomicAdd(&g_tc_prof[(S == 64 ? 8 : 0) + 5], 1ull);
@@ -911,7 +923,7 @@ __device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
   for (int h = 0; h < C::NP; h++) {
-    const int elem = h * C::EP + threadIdx.x / C::T;
+    const int elem = prod_elem<S>(h);
     if ((uint32_t)elem < valid) {
       const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + k * C::X);
       uint4* o = reinterpret_cast<uint4*>(dst + (size_t)elem * stride + k * C::X);
@@ -930,7 +942,7 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
   for (int h = 0; h < C::NP; h++) {
-    const int elem = h * C::EP + threadIdx.x / C::T;
+    const int elem = prod_elem<S>(h);
     uint32_t r[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
     load_const<X, C::T>(nn, Nmod);
@@ -940,7 +952,7 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
-  __syncthreads();
+  pair_sync();
 }
 
 // work row <- (row + s) mod N for every element (row, s < N)
@@ -952,7 +964,7 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
   for (int h = 0; h < C::NP; h++) {
-    const int elem = h * C::EP + threadIdx.x / C::T;
+    const int elem = prod_elem<S>(h);
     uint32_t r[X], a[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
     src_load<S>(a, s, elem, sW);
@@ -963,7 +975,7 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
-  __syncthreads();
+  pair_sync();
 }
 
 // ----------------------------------------------------------------------------- batched modexp
