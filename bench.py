@@ -37,8 +37,17 @@ KEY_SEED = 0xF1B0 + 2048
 ALPHA = 1.0
 SLOT_BITS = 32         # slots a multiple of 32 bits
 METRIC = "Paillier encrypt/decrypt/hom-add ops/sec at 2048-bit key, 1/2/4/8 B200"
+HBM_GBS = 6549.1  # MEASURED_PEAKS.json hbm_gbs (copy bandwidth), re-read below when the file is present
+try:
+    with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as _f:
+        HBM_GBS = float(__import__("json").load(_f).get("hbm_gbs", HBM_GBS))
+except (OSError, ValueError):
+    pass
 UNIT = "ops/s"
-PEAK_LP_PER_CLK_SM = 32  # IMAD.WIDE.U32(.X): half-rate FMA-heavy pipe (tools/imad_peak.cu)
+PEAK_LP_PER_CLK_SM = 32  # NOMINAL: IMAD.WIDE.U32(.X) at half rate on the FMA-heavy pipe (B300 guide: IMAD rt=2/SMSP)
+# measured ceilings of carry-chained IMAD.WIDE.U32.X sequences (tools/chain_lat.cu, profiles/r02_chain_lat.jsonl;
+# tools/imad_peak.cu, profiles/r01_imad_peak.jsonl): context for the nominal peak, not the denominator
+MEASURED_LP_PER_CLK_SM = {"chain_lat 2-chain, 16-64 warps/SM": 22.3, "imad_peak 1-chain, 64 warps/SM": 28.0}
 
 
 def parse():
@@ -358,15 +367,22 @@ def run_flb(args):
 
     # the other encryption path, timed once on the same batch (reported, not part of the step)
     other = "public" if args.encrypt == "keyholder" else "keyholder"
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    if other == "public":
-        flb.encrypt(pub, pt, seed=7, out=ct)
-    else:
-        flb.encrypt_crt(priv, pt, seed=7, out=ct)
-    e1.record()
-    torch.cuda.synchronize()
-    other_rate = ops_enc / world / (e0.elapsed_time(e1) * 1e-3)
+
+    def other_enc():
+        if other == "public":
+            flb.encrypt(pub, pt, seed=7, out=ct)
+        else:
+            flb.encrypt_crt(priv, pt, seed=7, out=ct)
+    other_enc()  # warm-up
+    other_ms = []
+    for _ in range(3):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        other_enc()
+        e1.record()
+        torch.cuda.synchronize()
+        other_ms.append(e0.elapsed_time(e1))
+    other_rate = ops_enc / world / (statistics.median(other_ms) * 1e-3)
 
     # roofline of the dominant kernel (encrypt): algorithmic limb products / its event time
     tc_on = os.environ.get("FLB_TC", "1") != "0"
@@ -421,9 +437,26 @@ def run_flb(args):
                     "imad_limb_products": dec_tc[1],
                     "imad_achieved": dec_tc[1] * rows / (phase["t_dec"] * 1e-3) / 1e12,
                     "frac": dec_tc[1] * rows / (phase["t_dec"] * 1e-3) / 1e12 / peak}
+    # the HBM-bound steps: bytes each moves per step / its event time (pack: float32 in, plaintext limbs
+    # out; unpack: plaintext limbs in, float32 out; reduce: CLIENTS ciphertexts in per row, one out)
+    add_lp = flb.op_cost(pub, "add")[1] // 2  # one Montgomery product (CIOS limb products) per reduce input
+    hbm = {
+        "pack": {"bytes": 4 * N_VALUES * CLIENTS + 4 * CLIENTS * rows * ptw, "ms": phase["t_pack"]},
+        "unpack": {"bytes": (r1 - r0 if world > 1 else rows) * ptw * 4 + 4 * my_values, "ms": phase["t_unpack"]},
+        "reduce": {"bytes": (CLIENTS + 1) * rows_p * ctw * 4 + 8 * (rows_p + 1 + CLIENTS * rows), "ms": phase["t_red"]},
+    }
+    for k, d in hbm.items():
+        d["GB_per_s"] = d["bytes"] / (d["ms"] * 1e-3) / 1e9 if d["ms"] > 0 else None
+        d["frac_of_measured_hbm"] = d["GB_per_s"] / HBM_GBS if d["GB_per_s"] else None
+    red_units = CLIENTS * rows
+    op_fracs = {
+        "encrypt (IMAD limb products of the dominant kernel)": achieved / peak,
+        "decrypt": dec_roof["frac"] if dec_roof else None,
+        "reduce (hom-add products, k_reduce CIOS)": add_lp * red_units / (phase["t_red"] * 1e-3) / 1e12 / peak,
+    }
     traffic = None
     tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json" if args.encrypt == "public" else
-                      ("encrypt_tc_traffic.json" if enc_tc else "encrypt_crt_traffic.json"))
+                      ("r02_encrypt_tc_traffic.json" if enc_tc else "encrypt_crt_traffic.json"))
     if os.path.exists(tp):
         try:
             with open(tp) as f:
@@ -525,11 +558,13 @@ def run_flb(args):
             "roofline": {"bound": "alu", "kernel": enc_kernel, "achieved": achieved, "peak": peak,
                          "unit": "T limb-products/s (IMAD.WIDE.U32 32x32->64, FMA-heavy pipe)",
                          "frac": achieved / peak, "traffic": traffic, "per_unit": per_unit,
-                         "peak_basis": "148 SM x 32 IMAD.WIDE/clk/SM x %.0f MHz (guide: IMAD rt=2/SMSP; "
-                                       "IMAD.WIDE half rate, measured tools/imad_peak.cu)" % sm_mhz_max,
+                         "peak_basis": "NOMINAL: 148 SM x 32 IMAD.WIDE/clk/SM x %.0f MHz (guide: IMAD rt=2/SMSP, "
+                                       "IMAD.WIDE half rate); nothing in MEASURED_PEAKS.json covers integer work" % sm_mhz_max,
+                         "measured_ceilings_lp_per_clk_sm": MEASURED_LP_PER_CLK_SM,
                          "tensor": tensor, "cios_equivalent_achieved": cios_eq,
                          "cios_equivalent_frac": cios_eq / peak},
             "decrypt_cost": {"mont_muls": dec_mm, "limb_products": dec_lp},
+            "op_roofline_fracs": op_fracs, "hbm_steps": hbm,
             "decrypt_roofline": dec_roof,
             "clocks": clk, "gpu_launches": launches_per_step * args.steps,
             "e2e": e2e, "cpu_baseline": cpu,
