@@ -575,7 +575,7 @@ def reduce_segments_host(pub: PublicKey, c, offsets, idx=None, max_segment_len: 
 
 
 OPS = {"encrypt": 0, "decrypt": 1, "add": 2, "reduce_input": 3, "encrypt_crt": 4, "encrypt_crt_tc": 5,
-       "decrypt_tc": 6, "encrypt_crt_tc_macs": 7, "decrypt_tc_macs": 8}
+       "decrypt_tc": 6, "encrypt_crt_tc_macs": 7, "decrypt_tc_macs": 8, "encrypt_tc": 9, "encrypt_tc_macs": 10}
 
 
 def op_cost(key, op: str) -> Tuple[int, int]:

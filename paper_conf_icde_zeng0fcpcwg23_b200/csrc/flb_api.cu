@@ -12,6 +12,36 @@ void set_last_error(const std::string& msg) { g_err = msg; }
 
 namespace {
 
+// Tensor-core Montgomery operands (flb_tc.cuh) for modulus N in an S-word frame, appended to blob:
+// extended Toeplitz K-slices Ext[r][kk] = V_(r - KB - kk) (bytes, zero outside [0, KB)) of
+// V = N' = -N^-1 mod R (2 KB rows) and V = N (3 KB rows), 32 bytes per row, in the K-major
+// core-matrix layout the MMA descriptors describe (KB = 4 S).
+void tc_operands(Blob& blob, const Limbs& N, uint32_t S, size_t* e1, size_t* e2) {
+  auto bytes_of = [](const Limbs& v, size_t nbytes) {
+    std::vector<uint8_t> b(nbytes, 0);
+    for (size_t i = 0; i < nbytes && i / 4 < v.size(); i++) b[i] = (uint8_t)(v[i / 4] >> (8 * (i % 4)));
+    return b;
+  };
+  auto ext = [&](const std::vector<uint8_t>& vb, uint32_t KB, uint32_t rows) {
+    std::vector<uint8_t> m((size_t)rows * 32, 0);
+    for (uint32_t r = 0; r < rows; r++)
+      for (uint32_t kk = 0; kk < 32; kk++) {
+        const int64_t d = (int64_t)r - KB - kk;
+        if (d >= 0 && d < (int64_t)KB) m[flb::tc::cm_off(r, kk, 2)] = vb[d];
+      }
+    std::vector<uint32_t> w(m.size() / 4, 0);
+    for (size_t i = 0; i < m.size(); i++) w[i / 4] |= (uint32_t)m[i] << (8 * (i % 4));
+    return blob.put_raw(w);
+  };
+  const uint32_t KB = 4 * S;
+  const Limbs Nf = H::resized(N, S);
+  Limbs np = H::resized(H::inv_mod_2k(Nf, S), S);  // N' = R - N^-1 (two's complement)
+  uint64_t cy = 1;
+  for (auto& w : np) { cy += (uint32_t)~w; w = (uint32_t)cy; cy >>= 32; }
+  *e1 = ext(bytes_of(np, KB), KB, 2 * KB);
+  *e2 = ext(bytes_of(Nf, KB), KB, 3 * KB);
+}
+
 flb_pub* make_pub(const Limbs& n_in) {
   auto* K = new flb_pub();
   K->nbits = (uint32_t)H::bits(n_in);
@@ -39,6 +69,13 @@ flb_pub* make_pub(const Limbs& n_in) {
   }
   K->o_RL = K->blob.put_raw(rl);
   K->o_sched = K->blob.put_raw(K->enc.ops);
+  K->o_one = K->blob.put_raw(std::vector<uint32_t>{1u, 0u, 0u, 0u});
+  // public-key encryption on the tensor cores (n^2 of 64 or 128 words; k_tc_exp starts from a table
+  // entry and needs at least one more schedule op)
+  if ((K->s == 64 || K->s == 128) && K->enc.ops.size() >= 2) {
+    tc_operands(K->blob, K->n2, K->s, &K->o_tcE1, &K->o_tcE2);
+    K->tc = true;
+  }
   return K;
 }
 
@@ -112,41 +149,14 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
       V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
     }
   }
-  // tensor-core Montgomery operands (flb_tc.cuh): extended Toeplitz K-slices
-  // Ext[r][kk] = V_(r - KB - kk) (bytes, zero outside [0, KB)) of V = N' = -N^-1 mod R (2 KB rows)
-  // and V = N (3 KB rows), 32 bytes per row, in the K-major core-matrix layout the MMA descriptors
-  // describe; for the P^2 moduli when sp is 32 or 64 (decryption, key-holder encryption stage 2)
-  // and for the half-frame P moduli when H is 32 or 64 (key-holder encryption stage 1)
+  // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 moduli when sp is 32, 64 or 128
+  // (decryption, key-holder encryption stage 2) and for the half-frame P moduli when H is 32 or 64
+  // (key-holder encryption stage 1)
   {
-    auto bytes_of = [](const Limbs& v, size_t nbytes) {
-      std::vector<uint8_t> b(nbytes, 0);
-      for (size_t i = 0; i < nbytes && i / 4 < v.size(); i++) b[i] = (uint8_t)(v[i / 4] >> (8 * (i % 4)));
-      return b;
-    };
-    auto ext = [&](const std::vector<uint8_t>& vb, uint32_t KB, uint32_t rows) {
-      std::vector<uint8_t> m((size_t)rows * 32, 0);
-      for (uint32_t r = 0; r < rows; r++)
-        for (uint32_t kk = 0; kk < 32; kk++) {
-          const int64_t d = (int64_t)r - KB - kk;
-          if (d >= 0 && d < (int64_t)KB) m[flb::tc::cm_off(r, kk, 2)] = vb[d];
-        }
-      std::vector<uint32_t> w(m.size() / 4, 0);
-      for (size_t i = 0; i < m.size(); i++) w[i / 4] |= (uint32_t)m[i] << (8 * (i % 4));
-      return V->blob.put_raw(w);
-    };
-    // (E1, E2) offsets for modulus N in an S-word frame
-    auto operands = [&](const Limbs& N, uint32_t S, size_t* e1, size_t* e2) {
-      const uint32_t KB = 4 * S;
-      const Limbs Nf = H::resized(N, S);
-      Limbs np = H::resized(H::inv_mod_2k(Nf, S), S);  // N' = R - N^-1 (two's complement)
-      uint64_t cy = 1;
-      for (auto& w : np) { cy += (uint32_t)~w; w = (uint32_t)cy; cy >>= 32; }
-      *e1 = ext(bytes_of(np, KB), KB, 2 * KB);
-      *e2 = ext(bytes_of(Nf, KB), KB, 3 * KB);
-    };
+    auto operands = [&](const Limbs& N, uint32_t S, size_t* e1, size_t* e2) { tc_operands(V->blob, N, S, e1, e2); };
     // (k_tc_exp starts from a table entry and needs at least one more schedule op: toy keys with
     // one-window exponents stay on the CIOS kernels)
-    if ((sp == 32 || sp == 64) && V->pr[0].sched.ops.size() >= 2 && V->pr[1].sched.ops.size() >= 2) {
+    if ((sp == 32 || sp == 64 || sp == 128) && V->pr[0].sched.ops.size() >= 2 && V->pr[1].sched.ops.size() >= 2) {
       for (int i = 0; i < 2; i++) operands(V->pr[i].P2, sp, &V->pr[i].o_tcE1, &V->pr[i].o_tcE2);
       V->tc = true;
     }
@@ -342,6 +352,14 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       *mont_muls = mm;
       return FLB_OK;
     }
+    case 9:     // public-key encryption, tensor-core kernel (k_tc_exp in the n^2 frame): IMAD limb products
+    case 10: {  // ... and its u8 MMA MACs
+      if (!P->tc) return fail(FLB_EUNSUPPORTED, "no tensor-core public-key path for this key");
+      const uint64_t mm = 1 + sched_mults(P->enc) + 2;
+      *mont_muls = mm;
+      *limb_products = op == 9 ? tc_imad_lp(s, mm, sched_squarings(P->enc)) : mm * tc_mma_macs(s);
+      return FLB_OK;
+    }
     case 2:
       *mont_muls = 2;
       *limb_products = 2 * cs;
@@ -478,17 +496,6 @@ static int pub_dev(const flb_pub* K, uint32_t** dev) { return const_cast<DevBlob
 
 extern "C" {
 
-int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* c,
-                size_t count, void* stream) {
-  if (!K || !m || !c) return fail(FLB_EINVAL, "null pointer");
-  if (count == 0) return FLB_OK;
-  uint32_t* dev;
-  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
-  if (rc) return rc;
-  if (debug_checks() && (rc = check_below(m, count, K->sp, dev + K->o_n, stream, "plaintexts m >= n"))) return rc;
-  FLB_DISPATCH_ENC(K->frame, run_encrypt, K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
-}
-
 // tensor-core Montgomery paths (flb_tc.cuh): on when the key has the operands; FLB_TC=0 selects
 // the CIOS kernels (read per call, so tests can compare both)
 static bool tc_enabled() {
@@ -503,6 +510,22 @@ static bool tc_dag_enabled() {
 static bool use_tc(const flb_priv* V) { return V->tc && tc_enabled(); }
 static bool use_tc_half(const flb_priv* V) { return V->tc_half && tc_enabled(); }
 
+int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t seed, uint64_t ctr0, uint32_t* c,
+                size_t count, void* stream) {
+  if (!K || !m || !c) return fail(FLB_EINVAL, "null pointer");
+  if (count == 0) return FLB_OK;
+  uint32_t* dev;
+  int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
+  if (rc) return rc;
+  if (debug_checks() && (rc = check_below(m, count, K->sp, dev + K->o_n, stream, "plaintexts m >= n"))) return rc;
+  if (K->tc && tc_enabled()) {
+    if (K->s == 128) return run_encrypt_pub_tc<128>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+    return run_encrypt_pub_tc<64>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+  }
+  FLB_DISPATCH_ENC(K->frame, run_encrypt, K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+}
+
+
 int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count, void* stream) {
   if (!V || !c || !m) return fail(FLB_EINVAL, "null pointer");
   if (count == 0) return FLB_OK;
@@ -516,6 +539,7 @@ int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count,
       return rc;
   }
   if (use_tc(V)) {
+    if (V->pub->sp == 128) return run_decrypt_tc<128>(V, dev, c, m, count, (cudaStream_t)stream);
     if (V->pub->sp == 64) return run_decrypt_tc<64>(V, dev, c, m, count, (cudaStream_t)stream);
     return run_decrypt_tc<32>(V, dev, c, m, count, (cudaStream_t)stream);
   }
@@ -557,9 +581,10 @@ int flb_add(const flb_pub* K, const uint32_t* c1, const uint32_t* c2, uint32_t* 
 int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, uint32_t words, int square,
                          void* stream) {
   if (!a || !b || !t || count > (uint32_t)flb::tc::kTileM) return fail(FLB_EINVAL, "null pointer or count > 128");
+  if (words == 128) return run_tc_debug_product<128>(a, b, t, count, square, (cudaStream_t)stream);
   if (words == 64) return run_tc_debug_product<64>(a, b, t, count, square, (cudaStream_t)stream);
   if (words == 32) return run_tc_debug_product<32>(a, b, t, count, square, (cudaStream_t)stream);
-  return fail(FLB_EINVAL, "words must be 32 or 64");
+  return fail(FLB_EINVAL, "words must be 32, 64 or 128");
 }
 
 int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
@@ -844,6 +869,7 @@ static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t
     rc = crt_pre_dispatch(V, dev, r, seed, ctr0, (uint32_t*)ys.p, count, st);
   if (rc) return rc;
   if (use_tc(V)) {
+    if (V->pub->sp == 128) return run_encrypt_crt_tc<128>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
     if (V->pub->sp == 64) return run_encrypt_crt_tc<64>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
     return run_encrypt_crt_tc<32>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
   }

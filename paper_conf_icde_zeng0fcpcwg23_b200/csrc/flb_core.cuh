@@ -111,6 +111,9 @@ struct flb_pub {
   H::Schedule enc;
   Blob blob;
   size_t o_n2 = 0, o_n = 0, o_R2 = 0, o_R1 = 0, o_nR = 0, o_RL = 0, o_sched = 0;
+  // tensor-core Montgomery operands for n^2 (flb_tc.cuh; ct_words in {64, 128}), and the integer 1
+  bool tc = false;
+  size_t o_tcE1 = 0, o_tcE2 = 0, o_one = 0;
   DevBlob dev;
 };
 
@@ -534,7 +537,7 @@ int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
   rc = tc_tiles(A, &tiles, &table);
   if (rc) return rc;
   if (tiles == 0) return FLB_OK;
-  const int grid = (int)std::min<uint64_t>((uint64_t)(2 * sms), tiles);  // two CTAs per SM
+  const int grid = (int)std::min<uint64_t>((uint64_t)(C::CTAS_PER_SM * sms), tiles);
   Scratch s_tab;
   rc = s_tab.alloc((size_t)grid * flb::tc::kTileM * (table + 1) * S * 4, st);
   if (rc) return rc;
@@ -633,6 +636,7 @@ void tc_stage2_args(const flb_priv* V, const uint32_t* dev, const uint32_t* m, c
     P.x_stride = V->H;
     P.x_words = V->H;
     P.m = m;
+    P.m_stride = P.m_words = V->pub->sp;
     P.nR = dev + R.o_nR;
     P.out = cpq + (size_t)i * count * S;
     P.count = count;
@@ -676,6 +680,65 @@ int run_encrypt_crt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m
   return tc_combine<S>(V, dev, cpq, c, count, st);
 }
 
+// r drawn on the device exactly as the CIOS encrypt kernel does (Philox, reading c4): [count][sp]
+inline int philox_fill(uint32_t sp, uint32_t nbits, uint64_t seed, uint64_t ctr0, size_t count, Scratch& s_r,
+                       cudaStream_t st) {
+  int rc = s_r.alloc((size_t)count * sp * 4, st);
+  if (rc) return rc;
+  int g;
+  switch (sp) {
+#define FLB_FILL(SPW)                                                                          \
+  case SPW:                                                                                    \
+    rc = grid_for<4>(flb::k_philox_fill<SPW / 4, 4>, count, &g); /* groups of 4 lanes (T a power of 2) */ \
+    if (rc) return rc;                                                                         \
+    flb::k_philox_fill<SPW / 4, 4><<<g, kBlock, 0, st>>>((uint32_t*)s_r.p, count, nbits, seed, ctr0); \
+    break;
+    FLB_FILL(32)
+    FLB_FILL(64)
+    FLB_FILL(96)
+    FLB_FILL(128)
+#undef FLB_FILL
+    default:
+      return fail(FLB_EUNSUPPORTED, "tensor-core path: unsupported plaintext frame");
+  }
+  FLB_LAUNCH_CHECK();
+  return FLB_OK;
+}
+
+// public-key encryption on the tensor cores (Eq. 3): c = (1 + m n) r^n mod n^2 in the
+// S = ct_words frame, every Montgomery product of the modexp with its reduction as u8 MMAs against
+// the Toeplitz operands of n^2 (one problem, k_tc_exp<S>)
+template <int S>
+int run_encrypt_pub_tc(const flb_pub* K, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                       uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  Scratch s_r;
+  if (!r) {
+    int rc = philox_fill(K->sp, K->nbits, seed, ctr0, count, s_r, st);
+    if (rc) return rc;
+    r = (const uint32_t*)s_r.p;
+  }
+  flb::tc::ExpArgs A{};
+  A.nprob = 1;
+  A.one = dev + K->o_one;
+  auto& P = A.pb[0];
+  P.N = dev + K->o_n2;
+  P.R2 = dev + K->o_R2;
+  P.R3 = nullptr;
+  P.E1 = dev + K->o_tcE1;
+  P.E2 = dev + K->o_tcE2;
+  P.sched = dev + K->o_sched;
+  P.sched_len = (int)K->enc.ops.size();
+  P.table = K->enc.table;
+  P.x = r;
+  P.x_stride = P.x_words = K->sp;
+  P.m = m;
+  P.m_stride = P.m_words = K->sp;
+  P.nR = dev + K->o_nR;
+  P.out = c;
+  P.count = count;
+  return launch_tc_exp<S>(A, st);
+}
+
 // key-holder stage 1 on the tensor cores: y_P = r^Q mod P in the H-word frame (both primes, one
 // launch); r drawn by k_philox_fill unless the caller passes it
 template <int HS>
@@ -683,24 +746,8 @@ int tc_stage1_args(const flb_priv* V, const uint32_t* dev, const uint32_t* r, ui
                    uint32_t* y, size_t count, cudaStream_t st, Scratch& s_r, flb::tc::ExpArgs& A) {
   const uint32_t sp = V->pub->sp;
   if (!r) {
-    int rc = s_r.alloc((size_t)count * sp * 4, st);
+    int rc = philox_fill(sp, V->pub->nbits, seed, ctr0, count, s_r, st);
     if (rc) return rc;
-    int g;
-    switch (sp) {
-#define FLB_FILL(SPW)                                                                          \
-  case SPW:                                                                                    \
-    rc = grid_for<4>(flb::k_philox_fill<SPW / 4, 4>, count, &g); /* groups of 4 lanes (T a power of 2) */ \
-    if (rc) return rc;                                                                         \
-    flb::k_philox_fill<SPW / 4, 4><<<g, kBlock, 0, st>>>((uint32_t*)s_r.p, count, V->pub->nbits, seed, ctr0); \
-    break;
-      FLB_FILL(64)
-      FLB_FILL(96)
-      FLB_FILL(128)
-#undef FLB_FILL
-      default:
-        return fail(FLB_EUNSUPPORTED, "tensor-core stage 1: unsupported plaintext frame");
-    }
-    FLB_LAUNCH_CHECK();
     r = (const uint32_t*)s_r.p;
   }
   A = flb::tc::ExpArgs{};
@@ -974,7 +1021,9 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
   EXT template int flb_rt::run_decrypt_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*, uint32_t*,       \
                                              size_t, cudaStream_t);                                              \
   EXT template int flb_rt::run_tc_debug_product<S>(const uint32_t*, const uint32_t*, uint32_t*, uint32_t, int,   \
-                                                   cudaStream_t);
+                                                   cudaStream_t);                                                 \
+  EXT template int flb_rt::run_encrypt_pub_tc<S>(const flb_pub*, const uint32_t*, const uint32_t*, const uint32_t*, \
+                                                 uint64_t, uint64_t, uint32_t*, size_t, cudaStream_t);
 #define FLB_TC_DAG_DECLS(EXT)                                                                                      \
   EXT template int flb_rt::run_encrypt_kh_dag<32, 64>(const flb_priv*, const uint32_t*, const uint32_t*,         \
                                                       const uint32_t*, uint64_t, uint64_t, uint32_t*, size_t,     \
@@ -987,6 +1036,7 @@ FLB_ENC_COMBOS(FLB_EXTERN_ENC)
 FLB_DEC_COMBOS(FLB_EXTERN_DEC)
 FLB_TC_DECLS(extern, 32)
 FLB_TC_DECLS(extern, 64)
+FLB_TC_DECLS(extern, 128)
 FLB_TC_DAG_DECLS(extern)
 #undef FLB_EXTERN_ENC
 #undef FLB_EXTERN_DEC

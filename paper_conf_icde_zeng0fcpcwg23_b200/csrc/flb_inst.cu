@@ -18,7 +18,10 @@ FLB_TC_DAG_DECLS()
 #endif
 #endif
 
-#if defined(FLB_INST_TC) && FLB_INST_TC == 64 && FLB_TC_PROF
+#if defined(FLB_INST_TC) && (FLB_INST_TC == 64 || FLB_INST_TC == 128) && FLB_TC_PROF
+#if FLB_INST_TC == 128
+#define flb_debug_tc_prof flb_debug_tc_prof128  // the k_tc_exp<128> object's own counters
+#endif
 // profiling builds only (FLB_NVCC_EXTRA=-DFLB_TC_PROF=1; not in include/): per-phase cycle totals of
 // thread 0 of the 2048-bit tensor-core Montgomery kernel (tools/tc_phases.py)
 extern "C" int flb_debug_tc_prof(uint64_t* out16, int reset) {

@@ -36,12 +36,12 @@ namespace flb {
 namespace tc {
 
 constexpr int kTileM = 128;     // elements per CTA tile (MMA M, TMEM lanes)
-constexpr int kThreads = 256;   // 8 warps; two CTAs per SM
-constexpr int kT = 4;           // lanes per element in the product phase at S >= 64 (S = 32: 2)
+constexpr int kThreads = 256;   // 8 warps; two CTAs per SM (one at S = 128)
+constexpr int kT = 4;           // lanes per element in the product phase at S = 64 (S = 32: 2, S = 128: 8)
 
 template <int S>
 struct Cfg {
-  static constexpr int T = S >= 64 ? kT : 2;       // lanes per element in the product phase
+  static constexpr int T = S >= 128 ? 8 : S >= 64 ? kT : 2;  // lanes per element in the product phase
   static constexpr int X = S / T;                  // limbs per lane (16)
   static constexpr int EP = kThreads / T;          // elements per product pass
   static constexpr int NP = kTileM / EP;           // product passes per tile
@@ -49,7 +49,8 @@ struct Cfg {
   static constexpr int KCH = KB / 16;              // 16-byte chunks per operand row
   static constexpr int QW = S / 2, QC = KB / 2;    // words / byte columns per normalising thread
   static constexpr int WROW = ((S + 4) / 4) % 2 == 1 ? S + 4 : S + 8;  // work row (words), /4 odd
-  static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB)
+  static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB) (S = 128: all 512 columns)
+  static constexpr int CTAS_PER_SM = S >= 128 ? 1 : 2;  // TMEM and shared memory per tile
   // dynamic shared memory carve-up (bytes)
   static constexpr int OFF_E1 = 0;                          // 2 KB rows x 32 bytes
   static constexpr int OFF_E2 = OFF_E1 + 2 * KB * 32;       // 3 KB rows x 32 bytes
@@ -57,7 +58,7 @@ struct Cfg {
   static constexpr int OFF_W = OFF_A + kTileM * KB;         // 128 work rows
   static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, 2 x uint4 per element
   static constexpr int SMEM = OFF_X + kTileM * 2 * 16;
-  static_assert(KB <= 256, "one MMA covers N <= 256 output columns");
+  static_assert(SMEM <= 227 * 1024, "shared memory per CTA");
   static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
 };
 
@@ -82,14 +83,19 @@ __device__ __forceinline__ uint32_t idesc_u8(int m, int n) {
   return (2u << 4) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(m >> 4) << 24);
 }
 
-// One K-slice MMA (A columns 32 ks .., B window starting at extended row r) into D columns [c0, c0 + n)
+// One K-slice MMA (A columns 32 ks .., B window starting at extended row r) into D columns [c0, c0 + n);
+// one instruction covers N <= 256 columns, so a wider slice (KB = 512 at S = 128) is issued in
+// 256-column pieces (the B window and the TMEM columns advance together)
 __device__ __forceinline__ void mma_slice(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext, uint32_t ks,
                                           uint32_t r, uint32_t c0, uint32_t n, uint32_t acc) {
   const uint64_t ad = smem_desc(sa + ks * 256u, kch * 128u);
-  const uint64_t bd = smem_desc(ext + (r >> 3) * 256u, 256u);
-  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-               "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
-               :: "r"(tmem_d + c0), "l"(ad), "l"(bd), "r"(idesc_u8(128, (int)n)), "r"(acc));
+  for (uint32_t o = 0; o < n; o += 256u) {
+    const uint32_t nn = n - o < 256u ? n - o : 256u;
+    const uint64_t bd = smem_desc(ext + ((r + o) >> 3) * 256u, 256u);
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
+                 :: "r"(tmem_d + c0 + o), "l"(ad), "l"(bd), "r"(idesc_u8(128, (int)nn)), "r"(acc));
+  }
 }
 
 // M1: D[:, j] = sum_K A[:, K] V[j - K] for j < KB (the low half of a Toeplitz product, V = N').
@@ -609,6 +615,94 @@ __device__ __forceinline__ void tc_square_product(const uint32_t (&a)[Cfg<S>::X]
     *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * cc) = make_uint4(q[4 * cc], q[4 * cc + 1], q[4 * cc + 2], q[4 * cc + 3]);
 }
 
+// Block squaring for eight lanes per element (S = 128, X = 16), the T = 4 scheme widened: lane k
+// computes its diagonal square a_k^2 (stored to its eighth t[2Xk, 2Xk + 2X)), the full cross blocks
+// a_k a_((k+d) mod 8) for d = 1, 2, 3 and half of the d = 4 block (row half k / 4 of a_(k%4) a_(k%4+4)),
+// each doubled and added in place at word X (k + l), in two disjoint-range phases per round (lanes
+// whose block does not wrap, then the ones that do; the two row halves of the d = 4 blocks).  Per
+// lane X (X+1)/2 + 3 X^2 + X^2/2 = 1032 limb products, S (S + 1) / 2 over the group.  The carry-out
+// (0..2) of every in-place addition lands at the word just past its range; each lane gathers, by
+// shuffles, the carries landing in its eighth and folds them in with one group pass and a ballot
+// carry-lookahead.
+template <int S, int SQ>
+__device__ __forceinline__ void tc_square_product_w(const uint32_t (&a)[Cfg<S>::X], int elem, uint8_t* sA,
+                                                    uint32_t* sW) {
+  constexpr int X = Cfg<S>::X, T = Cfg<S>::T, H = X / 2, HT = T / 2;
+  static_assert(T == 8, "eight lanes per element");
+  const int k = threadIdx.x % T;
+  {
+    uint32_t v[2 * X];
+    sqr_diag<X, SQ>(v, a);
+    __syncwarp();  // every lane of the group has read its a (it may come from the work row)
+#pragma unroll
+    for (int c = 0; c < X / 2; c++)
+      *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  }
+  uint32_t cw[HT];  // carry-out of each round's in-place addition
+#pragma unroll
+  for (int d = 1; d < HT; d++) {
+    uint32_t v[2 * X];
+    blk_prod<X, X, T>(v, a, a, (k + d) & (T - 1), false);
+    const bool wrap = k + d >= T;
+    const int w0 = X * (wrap ? 2 * k + d - T : 2 * k + d);
+    uint32_t c = 0;
+    __syncwarp();
+    if (!wrap) c = t_add_dbl<S, 2 * X>(sA, sW, elem, w0, v);
+    __syncwarp();
+    if (wrap) c = t_add_dbl<S, 2 * X>(sA, sW, elem, w0, v);
+    cw[d - 1] = c;
+  }
+  {
+    uint32_t M[X], v[X + H];
+    const int i = k & (HT - 1), hh = k / HT;
+#pragma unroll
+    for (int j = 0; j < X; j++) M[j] = __shfl_sync(FULL, a[j], i, T);
+    // rows [0, H) of a_(i+4) come from lane i + 4 (read by lane i); lane i + 4 takes its own rows [H, X)
+    blk_prod<X, H, T>(v, M, a, i + HT, hh == 1);
+    const int w0 = X * (2 * i + HT) + H * hh;
+    uint32_t c = 0;
+    __syncwarp();
+    if (hh == 0) c = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);
+    __syncwarp();
+    if (hh == 1) c = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);
+    __syncwarp();
+    cw[HT - 1] = c;
+  }
+  // the carries landing in this lane's eighth, at offsets 0, H, X, X + H (a carry past word 2S is 0:
+  // t = a^2 < 2^(64 S))
+  uint32_t at[4] = {0, 0, 0, 0};
+#pragma unroll
+  for (int r = 0; r < HT; r++) {
+#pragma unroll
+    for (int j = 0; j < T; j++) {
+      const uint32_t cj = __shfl_sync(FULL, cw[r], j, T);
+      int end;
+      if (r < HT - 1) {
+        const int d = r + 1;
+        end = X * ((j + d >= T ? 2 * j + d - T : 2 * j + d) + 2);
+      } else {
+        end = X * (2 * (j & (HT - 1)) + HT) + H * (j / HT) + X + H;
+      }
+      const int e = end / (2 * X), o = (end % (2 * X)) / H;
+      if (e < T && e == k) at[o] += cj;
+    }
+  }
+  uint32_t q[2 * X];
+#pragma unroll
+  for (int c = 0; c < X / 2; c++) {
+    const uint4 u = *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c);
+    q[4 * c] = u.x; q[4 * c + 1] = u.y; q[4 * c + 2] = u.z; q[4 * c + 3] = u.w;
+  }
+  const uint32_t cy = add_sparse_chain<2 * X, 0>(q, [&](int j) {
+    return j == 0 ? at[0] : j == H ? at[1] : j == X ? at[2] : j == X + H ? at[3] : 0u;
+  });
+  const uint32_t cc = group_carry<T>(cy != 0, all_ones<2 * X>(q), 0);
+  add_word_propagate<2 * X>(q, cc & 1u);
+#pragma unroll
+  for (int c = 0; c < X / 2; c++)
+    *t_chunk<S>(sA, sW, elem, 2 * X * k + 4 * c) = make_uint4(q[4 * c], q[4 * c + 1], q[4 * c + 2], q[4 * c + 3]);
+}
+
 // Block squaring for two lanes per element (S = 32, X = 16): lane k computes a_k^2 (X x X, stored to
 // t[2Xk, 2Xk + 2X)) and half of the cross block, a_0 a_1[H k, + H) (X x H, doubled, added at words
 // X + H k), 384 instead of 512 limb products per lane.  The two cross pieces overlap, so they are
@@ -677,10 +771,14 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
         tc_square_product_t2<S, SQ>(a, elem, sA, sW);
         continue;
       }
-    } else {
-      static_assert(S >= 64, "block squaring needs X x X blocks on 4 lanes");
+    } else if constexpr (T == 4) {
       if (sq) {
         tc_square_product<S, SQ>(a, elem, sA, sW);
+        continue;
+      }
+    } else {
+      if (sq) {
+        tc_square_product_w<S, SQ>(a, elem, sA, sW);
         continue;
       }
     }
@@ -999,7 +1097,8 @@ struct ExpProblem {
   int sched_len, table;
   const uint32_t* x;       // [count][x_stride]
   uint32_t x_stride, x_words;
-  const uint32_t* m;       // [count][S] or null
+  const uint32_t* m;       // [count][m_stride] (m_words limbs) or null
+  uint32_t m_stride, m_words;
   const uint32_t* nR;      // n R mod N (with m)
   uint32_t* out;           // [count][S]
   uint64_t count, tiles;
@@ -1076,7 +1175,8 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
   }
   if (P.m) {
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
-    tc_mont<S, SQ>(src_arr(P.m + e0 * S, S, S, nvalid), src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
+    tc_mont<S, SQ>(src_arr(P.m + e0 * P.m_stride, P.m_stride, P.m_words, nvalid), src_arr(P.nR, 0, S, kTileM), false,
+                   sm, P.N, phase);                         // m n
     tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
     tc_mont<S, SQ>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
   } else {
@@ -1112,7 +1212,7 @@ __device__ __forceinline__ void tc_cta_fini(uint32_t tmem) {
 }
 
 template <int S>
-__global__ void __launch_bounds__(kThreads, 2) k_tc_exp(const ExpArgs A) {
+__global__ void __launch_bounds__(kThreads, Cfg<S>::CTAS_PER_SM) k_tc_exp(const ExpArgs A) {
   using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;

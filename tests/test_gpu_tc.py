@@ -174,7 +174,7 @@ def test_tc_multi_tile_per_cta_both_problems():
     assert torch.equal(tc_d, m2)
 
 
-@pytest.mark.parametrize("words", [32, 64])
+@pytest.mark.parametrize("words", [32, 64, 128])
 @pytest.mark.parametrize("square", [0, 1, 2], ids=["general", "sqr_tri", "sqr_split"])
 def test_tc_product_phase_exact(words, square):
     """The tensor-core kernel's CUDA-core product phase (general row scan, or the block squaring
@@ -192,7 +192,7 @@ def test_tc_product_phase_exact(words, square):
         assert t[i] == want, (i, hex(t[i] ^ want))
 
 
-@pytest.mark.parametrize("words", [32, 64])
+@pytest.mark.parametrize("words", [32, 64, 128])
 @pytest.mark.parametrize("sq", [1, 2], ids=["tri", "split"])
 def test_tc_square_block_carries(words, sq):
     """Block squaring with triangular diagonal blocks (sqr_local: sum_{i<j} a_i a_j by lo/hi row
