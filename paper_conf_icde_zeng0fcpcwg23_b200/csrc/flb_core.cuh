@@ -543,7 +543,7 @@ int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
   if (rc) return rc;
   A.scratch = (uint32_t*)s_tab.p;
   A.tab_entries = table + 1;
-  flb::tc::k_tc_exp<S><<<grid, flb::tc::kThreads, C::SMEM, st>>>(A);
+  flb::tc::k_tc_exp<S><<<grid, C::THREADS, C::SMEM, st>>>(A);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }
@@ -601,11 +601,11 @@ int run_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint
   if (sq == 2) {
     FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 C::SMEM));
-    flb::tc::k_tc_debug_product<S, 2><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, 1);
+    flb::tc::k_tc_debug_product<S, 2><<<1, C::THREADS, C::SMEM, st>>>(a, b, t, count, 1);
   } else {
     FLB_CK(cudaFuncSetAttribute(flb::tc::k_tc_debug_product<S, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 C::SMEM));
-    flb::tc::k_tc_debug_product<S, 1><<<1, flb::tc::kThreads, C::SMEM, st>>>(a, b, t, count, sq);
+    flb::tc::k_tc_debug_product<S, 1><<<1, C::THREADS, C::SMEM, st>>>(a, b, t, count, sq);
   }
   FLB_LAUNCH_CHECK();
   return FLB_OK;

@@ -43,11 +43,18 @@ template <int S>
 struct Cfg {
   static constexpr int T = S >= 128 ? 8 : S >= 64 ? kT : 2;  // lanes per element in the product phase
   static constexpr int X = S / T;                  // limbs per lane (16)
-  static constexpr int EP = kThreads / T;          // elements per product pass
+  // threads per CTA: 8 warps (two CTAs per SM); at S = 128 (one CTA per SM: all TMEM) 16 warps, so
+  // the product phase keeps four warps per scheduler; the normalisation uses the first 8
+  static constexpr int THREADS = S >= 128 ? 512 : kThreads;
+  static constexpr int GW = THREADS / 128;         // warps per TMEM lane quadrant
+  static constexpr int EP = THREADS / T;           // elements per product pass
   static constexpr int NP = kTileM / EP;           // product passes per tile
   static constexpr int KB = 4 * S;                 // bytes of an S-word operand (MMA K and N)
   static constexpr int KCH = KB / 16;              // 16-byte chunks per operand row
-  static constexpr int QW = S / 2, QC = KB / 2;    // words / byte columns per normalising thread
+  // normalisation: each element's byte columns in NG groups, one thread each (the warps of its TMEM
+  // lane quadrant): 2 at 256 threads, 4 at S = 128 (512 threads); QW words / QC columns per thread
+  static constexpr int NG = THREADS / 128;
+  static constexpr int QW = S / NG, QC = KB / NG;
   static constexpr int WROW = ((S + 4) / 4) % 2 == 1 ? S + 4 : S + 8;  // work row (words), /4 odd
   static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB) (S = 128: all 512 columns)
   static constexpr int CTAS_PER_SM = S >= 128 ? 1 : 2;  // TMEM and shared memory per tile
@@ -56,8 +63,8 @@ struct Cfg {
   static constexpr int OFF_E2 = OFF_E1 + 2 * KB * 32;       // 3 KB rows x 32 bytes
   static constexpr int OFF_A = OFF_E2 + 3 * KB * 32;        // 128 x KB bytes (core matrices)
   static constexpr int OFF_W = OFF_A + kTileM * KB;         // 128 work rows
-  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, 2 x uint4 per element
-  static constexpr int SMEM = OFF_X + kTileM * 2 * 16;
+  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, NG x uint4 per element
+  static constexpr int SMEM = OFF_X + kTileM * NG * 16;
   static_assert(SMEM <= 227 * 1024, "shared memory per CTA");
   static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
 };
@@ -336,12 +343,14 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
 // threads); only the MMA issues, which read all 128 rows, need the whole CTA.
 template <int S>
 __device__ __forceinline__ int prod_elem(int h) {
-  constexpr int T = Cfg<S>::T;
+  constexpr int T = Cfg<S>::T, GW = Cfg<S>::GW;
   const int tid = threadIdx.x, warp = tid >> 5;
-  return 32 * (warp & 3) + h * (64 / T) + (warp >> 2) * (32 / T) + (tid & 31) / T;
+  return 32 * (warp & 3) + h * (32 * GW / T) + (warp >> 2) * (32 / T) + (tid & 31) / T;
 }
+// the warps of TMEM lane quadrant warp % 4 (2 at 256 threads: a warp pair; 4 at 512)
+template <int S>
 __device__ __forceinline__ void pair_sync() {
-  asm volatile("bar.sync %0, 64;" :: "r"(1 + ((threadIdx.x >> 5) & 3)) : "memory");
+  asm volatile("bar.sync %0, %1;" :: "r"(1 + ((threadIdx.x >> 5) & 3)), "n"(32 * Cfg<S>::GW) : "memory");
 }
 
 // ----------------------------------------------------------------------------- squaring product
@@ -499,12 +508,15 @@ __device__ __forceinline__ void sqr_diag(uint32_t (&v)[2 * X], const uint32_t (&
   if constexpr (SQ == 2) sqr_local_split<X>(v, a); else sqr_local<X>(v, a);
 }
 
-// address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work row
+// address of t's word w (w % 4 == 0) for element elem: words [0, S) in the sA row, [S, 2S) in the work
+// row.  With w % 4 == 0 the core-matrix offset of word w is cm_off(elem, 0) + 32 w (16-byte K chunks
+// 128 bytes apart), so a runtime w costs a shift-add and a select, the element bases are shared.
 template <int S>
 __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, int w) {
   using C = Cfg<S>;
-  return w < S ? reinterpret_cast<uint4*>(sA + cm_off(elem, 4u * w, C::KCH))
-               : reinterpret_cast<uint4*>(sW + elem * C::WROW + (w - S));
+  uint8_t* const a = sA + cm_off((uint32_t)elem, 0u, C::KCH) + 32u * (uint32_t)w;
+  uint8_t* const b = reinterpret_cast<uint8_t*>(sW + elem * C::WROW - S) + 4u * (uint32_t)w;
+  return reinterpret_cast<uint4*>(w < S ? a : b);
 }
 
 // t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2).  One carry
@@ -669,23 +681,27 @@ __device__ __forceinline__ void tc_square_product_w(const uint32_t (&a)[Cfg<S>::
     cw[HT - 1] = c;
   }
   // the carries landing in this lane's eighth, at offsets 0, H, X, X + H (a carry past word 2S is 0:
-  // t = a^2 < 2^(64 S))
+  // t = a^2 < 2^(64 S)).  Round d's carry from source lane j lands at word X (2j + d + 2) (no wrap)
+  // or X (2j + d - T + 2) (wrap), the half round's at X (2i + T/2 + 1) + H (hh + 1): so lane k takes
+  // round d's carry from lanes k - 1 - d/2 and k - (d - 7)/2 (d odd, at offset X) or k - (d - 6)/2
+  // (d even, at offset 0), and the half round's from lane k - 2 (hh = 0, at X + H) and lane k + 1
+  // (hh = 1, at 0) — the table enumerated and checked against the positions in DESIGN.md §6.
   uint32_t at[4] = {0, 0, 0, 0};
 #pragma unroll
-  for (int r = 0; r < HT; r++) {
-#pragma unroll
-    for (int j = 0; j < T; j++) {
-      const uint32_t cj = __shfl_sync(FULL, cw[r], j, T);
-      int end;
-      if (r < HT - 1) {
-        const int d = r + 1;
-        end = X * ((j + d >= T ? 2 * j + d - T : 2 * j + d) + 2);
-      } else {
-        end = X * (2 * (j & (HT - 1)) + HT) + H * (j / HT) + X + H;
-      }
-      const int e = end / (2 * X), o = (end % (2 * X)) / H;
-      if (e < T && e == k) at[o] += cj;
-    }
+  for (int d = 1; d < HT; d++) {
+    const int o = (d & 1) ? 2 : 0;
+    const int j1 = k - 1 - d / 2;
+    const int j2 = (d & 1) ? k - (d - 7) / 2 : k - (d - 6) / 2;
+    const uint32_t c1 = __shfl_sync(FULL, cw[d - 1], j1 & (T - 1), T);
+    const uint32_t c2 = __shfl_sync(FULL, cw[d - 1], j2 & (T - 1), T);
+    if (j1 >= 0 && j1 + d < T) at[o] += c1;
+    if (j2 >= T - d && j2 < T) at[o] += c2;
+  }
+  {
+    const uint32_t c1 = __shfl_sync(FULL, cw[HT - 1], (k - 2) & (T - 1), T);  // hh = 0, i = k - 2
+    const uint32_t c2 = __shfl_sync(FULL, cw[HT - 1], (k + 1) & (T - 1), T);  // hh = 1, i = k - 3
+    if (k >= 2 && k - 2 < HT) at[3] += c1;
+    if (k >= 3 && k - 3 < HT) at[0] += c2;
   }
   uint32_t q[2 * X];
 #pragma unroll
@@ -847,9 +863,11 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   }
   // normalisation: TMEM lane quadrant L = warp % 4 (elements 32L ..), column half g = warp / 4
   const int L = warp & 3, g = warp >> 2, i = 32 * L + (tid & 31);
+  const bool nw = true;  // every warp normalises: column group g of elements [32 L, 32 L + 32)
   const uint32_t lane_base = sm.tmem + ((uint32_t)(32 * L) << 16);
   uint32_t* row = sW + i * C::WROW;
-  uint4* xch = reinterpret_cast<uint4*>(sm.base + C::OFF_X) + i * 2;
+  uint4* xch = reinterpret_cast<uint4*>(sm.base + C::OFF_X) + i * C::NG;
+  constexpr int NG = C::NG;
   uint2 ttop = make_uint2(0, 0);
   if (g == 0) ttop = *reinterpret_cast<const uint2*>(sA + cm_off(i, KB - 8, KCH));  // t_lo bytes KB-8 ..
   mbar_wait(sm.mbar, phase);
@@ -875,8 +893,16 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     const uint64_t ov = (x.z != 0u && (((uint64_t)x.y + cin) >> 32) != 0) ? 1u : 0u;
     return (uint64_t)x.x + ov;
   };
+  // carry into column group gg (the prefix over the groups below it)
+  auto carry_into = [&](int gg) {
+    uint64_t c = 0;
+#pragma unroll
+    for (int h = 0; h < NG - 1; h++)
+      if (h < gg) c = carry_out(h, c);
+    return c;
+  };
   // ---- N1: q = D1 mod R
-  {
+  if (nw) {
     NormState ns;
 #pragma unroll
     for (int c0 = 0; c0 < QC; c0 += 32) {
@@ -887,11 +913,14 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
     publish(ns.carry_out_end());
   }
-  pair_sync();  // carries published (D1 drained before M2: the CTA barrier below)
-  if (g == 1) add_in(carry_out(0, 0));
+  pair_sync<S>();  // carries published (D1 drained before M2: the CTA barrier below)
+  if (nw) {
+    if (g > 0) add_in(carry_into(g));
 #pragma unroll
-  for (int c = 0; c < QW / 4; c++)
-    *reinterpret_cast<uint4*>(sA + cm_off(i, g * QC + 16 * c, KCH)) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+    for (int c = 0; c < QW / 4; c++)
+      *reinterpret_cast<uint4*>(sA + cm_off(i, g * QC + 16 * c, KCH)) =
+          make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+  }
   fence_async_smem();
   tc_before_sync();
   __syncthreads();
@@ -909,7 +938,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- F: u = t_hi + high(q N) + c'.  t_lo + (q N mod R) = c' R exactly; with W = the 8 byte
   // columns below KB of t + q N (as an integer over those columns) and Z the rest
   // (< 2^(8(KB-8)+26)), c' R = W 2^(8(KB-8)) + Z, so c' = ceil(W / 2^64).  Half 0 starts with c'.
-  {
+  if (nw) {
     uint64_t carry = 0;
     if (g == 0) {
       uint32_t bc[8];
@@ -924,10 +953,10 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
     NormState ns;
     ns.hprev = (uint32_t)carry;  // < 2^20
-    // this half's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; half 1's last 8 columns
-    // (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
+    // this group's columns KB + g QC + c, i.e. D2 columns 8 + g QC + c; the last group's last 8
+    // columns (2KB-8 .. 2KB-1) are outside D2: the 7 top columns of q N from its top 8 bytes and N's
     uint32_t top[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    if (g == 1) {
+    if (g == NG - 1) {
       const uint2 qt2 = *reinterpret_cast<const uint2*>(sA + cm_off(i, KB - 8, KCH));
       const uint2 nt2 = __ldg(reinterpret_cast<const uint2*>(Nmod + S - 2));
       uint32_t qt[8], nt[8];
@@ -951,15 +980,15 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       if (c0 + 32 < QC) {
         tmem_ld32(lane_base + col, cv);
       } else {
-        // last chunk of the half: D2 columns col .. col+23 always exist; col+24 .. col+31 exist
-        // for half 0 only (half 1's are the top columns)
+        // last chunk of the group: D2 columns col .. col+23 always exist; col+24 .. col+31 exist
+        // for all but the last group (whose are the top columns)
         tmem_ld16(lane_base + col, cv);
         tmem_ld8(lane_base + col + 16u, cv + 16);
         uint32_t t8[8];
-        tmem_ld8(lane_base + (g == 0 ? col + 24u : 0u), t8);  // uniform per warp; unused for half 1
+        tmem_ld8(lane_base + (g < NG - 1 ? col + 24u : 0u), t8);  // uniform per warp; unused for the last
         tmem_wait();
 #pragma unroll
-        for (int j = 0; j < 8; j++) cv[24 + j] = g == 0 ? t8[j] : top[j];
+        for (int j = 0; j < 8; j++) cv[24 + j] = g < NG - 1 ? t8[j] : top[j];
       }
       tmem_wait();
       const uint4 h0 = reinterpret_cast<const uint4*>(row + g * QW + c0 / 4)[0];
@@ -969,13 +998,14 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
     publish(ns.carry_out_end());
   }
-  pair_sync();
-  const uint64_t c1 = carry_out(0, 0);
-  const uint64_t ovf = carry_out(1, c1);  // bit above S words (u < 2N < 2R)
-  if (g == 1) add_in(c1);
-  // u - N over this half: local borrow and zero-difference flag
+  pair_sync<S>();
+  uint64_t ovf = 0;
   uint32_t d[QW];
-  {
+  if (nw) {
+    const uint64_t cg = carry_into(g);
+    ovf = carry_out(NG - 1, carry_into(NG - 1));  // bit above S words (u < 2N < 2R)
+    if (g > 0) add_in(cg);
+    // u - N over this group: local borrow and zero-difference flag
     uint32_t br = 0, nzd = 0;
     uint32_t nn[QW];
 #pragma unroll
@@ -991,13 +1021,18 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     for (int w = 0; w < QW; w++) nzd |= d[w];
     xch[g].w = br | (nzd == 0u ? 2u : 0u);
   }
-  pair_sync();
-  {
-    const uint32_t f0 = xch[0].w, f1 = xch[1].w;
-    const uint32_t b1 = f0 & 1u;                          // borrow into half 1
-    const uint32_t bout = (f1 & 1u) | ((f1 >> 1) & b1);    // borrow out of the top
+  pair_sync<S>();
+  if (nw) {
+    // borrow into each group: b_(h+1) = borrow_h | (zero_h & b_h); bout = the borrow out of the top
+    uint32_t bin = 0, bout = 0;
+#pragma unroll
+    for (int h = 0; h < NG; h++) {
+      if (h == g) bin = bout;
+      const uint32_t f = xch[h].w;
+      bout = (f & 1u) | ((f >> 1) & bout);
+    }
     if (ovf != 0 || bout == 0) {                           // u >= N: take u - N
-      v[0] = sub_cc(d[0], g == 1 ? b1 : 0u);
+      v[0] = sub_cc(d[0], bin);
 #pragma unroll
       for (int w = 1; w < QW; w++) v[w] = subc_cc(d[w], 0u);
     }
@@ -1006,7 +1041,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
       reinterpret_cast<uint4*>(row + g * QW)[c] = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
   }
   tc_before_sync();
-  pair_sync();  // the pair's rows are final (the next product / row op of these elements is the pair's)
+  pair_sync<S>();  // the pair's rows are final (the next product / row op of these elements is the pair's)
   TC_MARK(4);
 #if FLB_TC_PROF
   if (threadIdx.x == 0) atomicAdd(&g_tc_prof[(S == 64 ? 8 : 0) + 5], 1ull);
@@ -1050,7 +1085,7 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
-  pair_sync();
+  pair_sync<S>();
 }
 
 // work row <- (row + s) mod N for every element (row, s < N)
@@ -1073,7 +1108,7 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
-  pair_sync();
+  pair_sync<S>();
 }
 
 // ----------------------------------------------------------------------------- batched modexp
@@ -1119,8 +1154,8 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
   const uint4* s2 = reinterpret_cast<const uint4*>(P.E2);
   uint4* d1 = reinterpret_cast<uint4*>(smem + C::OFF_E1);
   uint4* d2 = reinterpret_cast<uint4*>(smem + C::OFF_E2);
-  for (int i = threadIdx.x; i < 2 * KB * 32 / 16; i += kThreads) d1[i] = __ldg(s1 + i);
-  for (int i = threadIdx.x; i < 3 * KB * 32 / 16; i += kThreads) d2[i] = __ldg(s2 + i);
+  for (int i = threadIdx.x; i < 2 * KB * 32 / 16; i += C::THREADS) d1[i] = __ldg(s1 + i);
+  for (int i = threadIdx.x; i < 3 * KB * 32 / 16; i += C::THREADS) d2[i] = __ldg(s2 + i);
   fence_async_smem();
 }
 
@@ -1212,7 +1247,7 @@ __device__ __forceinline__ void tc_cta_fini(uint32_t tmem) {
 }
 
 template <int S>
-__global__ void __launch_bounds__(kThreads, Cfg<S>::CTAS_PER_SM) k_tc_exp(const ExpArgs A) {
+__global__ void __launch_bounds__(Cfg<S>::THREADS, Cfg<S>::CTAS_PER_SM) k_tc_exp(const ExpArgs A) {
   using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;
@@ -1308,7 +1343,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, co
 
 // debug: the product phase alone (t = a b, or a^2 when sq) for up to 128 elements -> t [count][2S]
 template <int S, int SQ>
-__global__ void __launch_bounds__(kThreads, 1) k_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t,
+__global__ void __launch_bounds__(Cfg<S>::THREADS, 1) k_tc_debug_product(const uint32_t* a, const uint32_t* b, uint32_t* t,
                                                                   uint32_t count, int sq) {
   using C = Cfg<S>;
   extern __shared__ __align__(1024) uint8_t smem[];
@@ -1316,7 +1351,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_tc_debug_product(const uint32_t
   uint32_t* sW = reinterpret_cast<uint32_t*>(smem + C::OFF_W);
   tc_product<S, SQ>(src_arr(a, S, S, count), src_arr(b, S, S, count), sq != 0, sA, sW);
   __syncthreads();
-  for (uint32_t i = threadIdx.x; i < count * 2 * S; i += kThreads) {
+  for (uint32_t i = threadIdx.x; i < count * 2 * S; i += C::THREADS) {
     const uint32_t e = i / (2 * S), w = i % (2 * S);
     t[i] = w < (uint32_t)S ? *reinterpret_cast<const uint32_t*>(sA + cm_off(e, 4u * w, C::KCH)) : sW[e * C::WROW + w - S];
   }
