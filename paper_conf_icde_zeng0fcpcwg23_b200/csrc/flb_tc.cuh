@@ -92,16 +92,21 @@ __device__ __forceinline__ uint32_t idesc_u8(int m, int n) {
 
 // One K-slice MMA (A columns 32 ks .., B window starting at extended row r) into D columns [c0, c0 + n);
 // one instruction covers N <= 256 columns, so a wider slice (KB = 512 at S = 128) is issued in
-// 256-column pieces (the B window and the TMEM columns advance together)
-__device__ __forceinline__ void mma_slice(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext, uint32_t ks,
-                                          uint32_t r, uint32_t c0, uint32_t n, uint32_t acc) {
-  const uint64_t ad = smem_desc(sa + ks * 256u, kch * 128u);
-  for (uint32_t o = 0; o < n; o += 256u) {
-    const uint32_t nn = n - o < 256u ? n - o : 256u;
-    const uint64_t bd = smem_desc(ext + ((r + o) >> 3) * 256u, 256u);
-    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-                 "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
-                 :: "r"(tmem_d + c0 + o), "l"(ad), "l"(bd), "r"(idesc_u8(128, (int)nn)), "r"(acc));
+// 256-column pieces (the B window and the TMEM columns advance together).  KB is a template
+// parameter so the slice loops unroll and every (r, c0, n) is a constant.
+template <int KB>
+__device__ __forceinline__ void mma_slice(uint32_t tmem_d, uint32_t sa, uint32_t ext, uint32_t ks, uint32_t r,
+                                          uint32_t c0, uint32_t n, uint32_t acc) {
+  const uint64_t ad = smem_desc(sa + ks * 256u, (uint32_t)KB * 8u);
+#pragma unroll
+  for (uint32_t o = 0; o < (uint32_t)KB; o += 256u) {
+    if (o < n) {
+      const uint32_t nn = n - o < 256u ? n - o : 256u;
+      const uint64_t bd = smem_desc(ext + ((r + o) >> 3) * 256u, 256u);
+      asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                   "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}"
+                   :: "r"(tmem_d + c0 + o), "l"(ad), "l"(bd), "r"(idesc_u8(128, (int)nn)), "r"(acc));
+    }
   }
 }
 
@@ -109,19 +114,21 @@ __device__ __forceinline__ void mma_slice(uint32_t tmem_d, uint32_t sa, uint32_t
 // Slice ks (K in [32 ks, 32 ks + 32)) adds nothing to the columns j < 32 ks, so it is issued for
 // columns [32 ks, KB) only (its B window then starts at extended row KB for every ks): 36/64 of the
 // full MACs.  Slice 0 (all columns) initialises D.
-__device__ __forceinline__ void mma_toeplitz_lo(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext) {
-  const uint32_t KB = kch * 16u;
-  for (uint32_t ks = 0; ks < kch / 2; ks++) mma_slice(tmem_d, sa, kch, ext, ks, KB, 32u * ks, KB - 32u * ks, ks > 0);
+template <int KB>
+__device__ __forceinline__ void mma_toeplitz_lo(uint32_t tmem_d, uint32_t sa, uint32_t ext) {
+#pragma unroll
+  for (uint32_t ks = 0; ks < (uint32_t)KB / 32u; ks++)
+    mma_slice<KB>(tmem_d, sa, ext, ks, KB, 32u * ks, KB - 32u * ks, ks > 0);
 }
 // M2: D[:, j] = sum_K A[:, K] V[KB - 8 + j - K] (V = N, zero at index >= KB) for j < KB: slice ks
 // reaches only the columns j < 32 ks + 40, so it is issued for [0, min(KB, 32 ks + 48)); the widest
 // slice goes first and initialises D.
-__device__ __forceinline__ void mma_toeplitz_hi(uint32_t tmem_d, uint32_t sa, uint32_t kch, uint32_t ext) {
-  const uint32_t KB = kch * 16u;
-  for (int ks = (int)kch / 2 - 1; ks >= 0; ks--) {
-    const uint32_t n = min(KB, 32u * (uint32_t)ks + 48u);
-    mma_slice(tmem_d, sa, kch, ext, (uint32_t)ks, 2u * KB - 8u - 32u * (uint32_t)ks, 0u, n,
-              ks != (int)kch / 2 - 1);
+template <int KB>
+__device__ __forceinline__ void mma_toeplitz_hi(uint32_t tmem_d, uint32_t sa, uint32_t ext) {
+#pragma unroll
+  for (int ks = KB / 32 - 1; ks >= 0; ks--) {
+    const uint32_t n = min((uint32_t)KB, 32u * (uint32_t)ks + 48u);
+    mma_slice<KB>(tmem_d, sa, ext, (uint32_t)ks, 2u * KB - 8u - 32u * (uint32_t)ks, 0u, n, ks != KB / 32 - 1);
   }
 }
 
@@ -858,7 +865,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- M1: q columns [0, KB)
   if (tid == 0) {
     tc_after_sync();
-    mma_toeplitz_lo(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E1));
+    mma_toeplitz_lo<KB>(sm.tmem, smem_u32(sA), smem_u32(sm.base + C::OFF_E1));
     mma_commit(sm.mbar);
   }
   // normalisation: TMEM lane quadrant L = warp % 4 (elements 32L ..), column half g = warp / 4
@@ -927,7 +934,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- M2: q N columns [KB-8, 2KB-8) into D2 = TMEM [0, KB)
   if (tid == 0) {
     tc_after_sync();
-    mma_toeplitz_hi(sm.tmem, smem_u32(sA), KCH, smem_u32(sm.base + C::OFF_E2));
+    mma_toeplitz_hi<KB>(sm.tmem, smem_u32(sA), smem_u32(sm.base + C::OFF_E2));
     mma_commit(sm.mbar);
   }
   TC_MARK(2);
