@@ -601,12 +601,26 @@ def run_other(args):
     """C1, C3, C4, C5 on one GPU (BASELINE.json configs[0], [2], [3], [4])."""
     import numpy as np
     import torch
+    import torch.distributed as dist
     import paper_conf_icde_zeng0fcpcwg23_b200 as flb
     import synthetic
-    torch.cuda.set_device(0)
-    dev = torch.device("cuda", 0)
     wl = args.workload
-    clk = ClockSampler(0)
+    world = int(os.environ.get("WORLD_SIZE", "1")) if wl == "c5" else 1
+    rank = int(os.environ.get("RANK", "0")) if world > 1 else 0
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:  # C5 shards by ciphertext (weak scaling); the other configs run on one GPU
+        torch.cuda.set_device(local % torch.cuda.device_count())
+        backend = os.environ.get("FLB_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local % torch.cuda.device_count()))
+        else:
+            dist.init_process_group(backend)
+    elif int(os.environ.get("RANK", "0")) != 0:
+        return 0  # C1/C3/C4 are single-GPU configs: the other ranks have nothing to do
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    clk = ClockSampler(torch.cuda.current_device())
     res = {"metric": METRIC, "unit": UNIT, "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
            "dtype": "u32-limb bigint (+f64 codec)", "data": "synthetic"}
@@ -618,10 +632,14 @@ def run_other(args):
             step(s)
         torch.cuda.synchronize()
         ev.clear()
+        if world > 1:
+            dist.barrier()
         for s in range(args.steps):
             flush.zero_()
             step(100 + s)
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         return _phases(ev, names, args.steps)
 
     ev, mark = _timer()
@@ -749,7 +767,7 @@ def run_other(args):
     elif wl == "c5":
         per = {}
         for bits in (1024, 2048, 3072, 4096):
-            M = args.c5_ops or ((1 << 20) if bits <= 2048 else (1 << 18))
+            M = args.c5_ops or ((1 << 20) if bits <= 2048 else (1 << 18))  # per rank (weak scaling)
             pub, priv = flb.keygen(bits, 0xF1B0 + bits)
             p, q, n = priv.export()
             base = synthetic.ints_to_limbs(synthetic.uniform_below(n, 256, 5 + bits), pub.pt_words).view(np.int32)
@@ -761,9 +779,9 @@ def run_other(args):
 
             def step(s):
                 mark("t0")
-                flb.encrypt(pub, m, seed=s, out=c)
+                flb.encrypt(pub, m, seed=s, ctr0=rank * M, out=c)
                 mark("enc")
-                flb.encrypt_crt(priv, m, seed=s, out=o)
+                flb.encrypt_crt(priv, m, seed=s, ctr0=rank * M, out=o)
                 mark("enc_crt")
                 flb.decrypt(priv, c, out=dm)
                 mark("dec")
@@ -771,37 +789,49 @@ def run_other(args):
                 mark("add")
             names = ["t0", "enc", "enc_crt", "dec", "add"]
             ms, ph = run_steps(step, names)
+            if world > 1:  # max over ranks of every phase (weak scaling: each rank its own batch)
+                t = torch.tensor([ph[k] for k in names[1:]], dtype=torch.float64,
+                                 device=dev if dist.get_backend() == "nccl" else "cpu")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                ph = {k: float(t[i]) for i, k in enumerate(names[1:])}
             lp = {k: flb.op_cost(priv if k in ("decrypt", "encrypt_crt") else pub, k)[1]
                   for k in ("encrypt", "encrypt_crt", "decrypt", "add")}
-            # tensor-core kernels: count the IMAD-pipe work they actually issue (op_cost 5/6)
-            acct = {"encrypt_crt": "cios", "decrypt": "cios"}
+            # tensor-core kernels: count the IMAD-pipe work they actually issue (op_cost 5/6/9)
+            acct = {"encrypt": "cios", "encrypt_crt": "cios", "decrypt": "cios"}
             if os.environ.get("FLB_TC", "1") != "0":
-                for k, tk in (("encrypt_crt", "encrypt_crt_tc"), ("decrypt", "decrypt_tc")):
+                for k, tk, key in (("encrypt_crt", "encrypt_crt_tc", priv), ("decrypt", "decrypt_tc", priv),
+                                   ("encrypt", "encrypt_tc", pub)):
                     try:
-                        lp[k] = flb.op_cost(priv, tk)[1]
+                        lp[k] = flb.op_cost(key, tk)[1]
                         acct[k] = "tensor-core (IMAD-pipe limb products of t = a b; reduction on tcgen05)"
                     except flb.FlbError:
                         pass
             peak = 148 * PEAK_LP_PER_CLK_SM * 1965e6
+            W = world * M  # ops over all ranks
             per[str(bits)] = {
-                "batch": M,
-                "encrypt_per_s": M / (ph["enc"] * 1e-3), "encrypt_keyholder_per_s": M / (ph["enc_crt"] * 1e-3),
-                "decrypt_per_s": M / (ph["dec"] * 1e-3), "add_per_s": M / (ph["add"] * 1e-3),
-                "frac_roofline": {"encrypt": lp["encrypt"] * M / (ph["enc"] * 1e-3) / peak,
-                                  "encrypt_keyholder": lp["encrypt_crt"] * M / (ph["enc_crt"] * 1e-3) / peak,
-                                  "decrypt": lp["decrypt"] * M / (ph["dec"] * 1e-3) / peak,
-                                  "add": lp["add"] * M / (ph["add"] * 1e-3) / peak},
+                "batch_per_rank": M,
+                "encrypt_per_s": W / (ph["enc"] * 1e-3), "encrypt_keyholder_per_s": W / (ph["enc_crt"] * 1e-3),
+                "decrypt_per_s": W / (ph["dec"] * 1e-3), "add_per_s": W / (ph["add"] * 1e-3),
+                "frac_roofline": {"encrypt": lp["encrypt"] * W / (ph["enc"] * 1e-3) / peak / world,
+                                  "encrypt_keyholder": lp["encrypt_crt"] * W / (ph["enc_crt"] * 1e-3) / peak / world,
+                                  "decrypt": lp["decrypt"] * W / (ph["dec"] * 1e-3) / peak / world,
+                                  "add": lp["add"] * W / (ph["add"] * 1e-3) / peak / world},
                 "imad_accounting": acct}
             del c, o, dm, m
         v = per["2048"]
         res.update(value=3.0 / (1 / v["encrypt_per_s"] + 1 / v["decrypt_per_s"] + 1 / v["add_per_s"]),
                    ms_per_step=None, per_key=per,
+                   n_gpus=world, scaling="weak",
                    config={"workload": "C5 key sweep 1024/2048/3072/4096: encrypt (public and key-holder), "
-                                       "decrypt, add on uniform m < n; batch 1,048,576 (1024/2048) and 262,144 "
-                                       "(3072/4096) per op instead of 16M (time budget)",
+                                       "decrypt, add on uniform m < n; per rank batch 1,048,576 (1024/2048) and "
+                                       "262,144 (3072/4096) per op instead of 16M (time budget; --c5-ops 16777216 "
+                                       "runs the full batch), shard by ciphertext over %d rank(s)" % world,
                            "value_definition": "2048-bit enc/dec/add mix: 3 / sum of per-op seconds"})
     res["clocks"] = clk.stop()
-    print(json.dumps(res), flush=True)
+    if rank == 0:
+        print(json.dumps(res), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
     return 0
 
 
