@@ -521,9 +521,14 @@ __device__ __forceinline__ void sqr_diag(uint32_t (&v)[2 * X], const uint32_t (&
 template <int S>
 __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, int w) {
   using C = Cfg<S>;
-  uint8_t* const a = sA + cm_off((uint32_t)elem, 0u, C::KCH) + 32u * (uint32_t)w;
-  uint8_t* const b = reinterpret_cast<uint8_t*>(sW + elem * C::WROW - S) + 4u * (uint32_t)w;
-  return reinterpret_cast<uint4*>(w < S ? a : b);
+  if constexpr (S >= 128) {
+    uint8_t* const a = sA + cm_off((uint32_t)elem, 0u, C::KCH) + 32u * (uint32_t)w;
+    uint8_t* const b = reinterpret_cast<uint8_t*>(sW + elem * C::WROW - S) + 4u * (uint32_t)w;
+    return reinterpret_cast<uint4*>(w < S ? a : b);
+  } else {  // (measured: the select-free form below issues fewer instructions at S <= 64)
+    return w < S ? reinterpret_cast<uint4*>(sA + cm_off(elem, 4u * w, C::KCH))
+                 : reinterpret_cast<uint4*>(sW + elem * C::WROW + (w - S));
+  }
 }
 
 // t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2).  One carry
