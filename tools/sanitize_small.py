@@ -1,4 +1,10 @@
-"""Small runs of every kernel for compute-sanitizer (memcheck / racecheck / synccheck / initcheck)."""
+"""Small runs of every kernel for compute-sanitizer (memcheck / racecheck / synccheck / initcheck).
+
+    python tools/sanitize_small.py          # 37-element batches of every op (toy16 / 1024 / 2048 / 4096)
+    python tools/sanitize_small.py dag      # + a 20,000-element key-holder encryption at 2048 bits: 157
+                                            #   stage-1 and 157 stage-2 tiles per prime on 296 CTAs, so
+                                            #   stage-2 tiles wait on flags set by other CTAs
+"""
 import os
 import sys
 
@@ -11,7 +17,8 @@ import synthetic  # noqa: E402
 from tests.helpers import golden_keys  # noqa: E402
 
 K = golden_keys()
-for name in ("toy16", "1024", "2048"):
+dag = len(sys.argv) > 1 and sys.argv[1] == "dag"
+for name in ("toy16", "1024", "2048", "4096"):
     p, q = K[name]
     pub, priv = flb.key_from_primes(p, q)
     n = p * q
@@ -34,4 +41,23 @@ for name in ("toy16", "1024", "2048"):
         us = flb.unpack_sums(pub, cd, pt, 100)
     torch.cuda.synchronize()
     assert torch.equal(d, m) and torch.equal(c, c2)
+# Table I fundamentals (csrc/flb_mp.cu)
+a = torch.randint(-2**31, 2**31 - 1, (37, 33), dtype=torch.int32).cuda()
+b = torch.randint(-2**31, 2**31 - 1, (37, 33), dtype=torch.int32).cuda()
+flb.mp_add(a, b)
+flb.mp_sub(a, b)
+flb.mp_mul(a, b)
+flb.mp_divmod(a, b)
+b[:, 0] |= 1
+flb.mp_mod_inv(a, b)
+torch.cuda.synchronize()
+if dag:
+    p, q = K["2048"]
+    pub, priv = flb.key_from_primes(p, q)
+    M = 20000
+    m = torch.from_numpy(synthetic.ints_to_limbs(synthetic.uniform_below(p * q, 64, 2), pub.pt_words)
+                         .view(np.int32)).cuda().repeat(M // 64 + 1, 1)[:M].contiguous()
+    c2 = flb.encrypt_crt(priv, m, seed=5)
+    torch.cuda.synchronize()
+    assert torch.equal(flb.decrypt(priv, c2), m)
 print("sanitize run ok")
