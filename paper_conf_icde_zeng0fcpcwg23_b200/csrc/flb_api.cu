@@ -42,6 +42,17 @@ void tc_operands(Blob& blob, const Limbs& N, uint32_t S, size_t* e1, size_t* e2)
   *e2 = ext(bytes_of(Nf, KB), KB, 3 * KB);
 }
 
+// largest sliding window of the key's exponent schedules; FLB_WMAX (1..7, read at key
+// import) is a measurement knob for the window-table footprint
+static int sched_wmax() {
+  static const int w = [] {
+    const char* e = getenv("FLB_WMAX");
+    const int v = e ? atoi(e) : 7;
+    return v < 1 ? 1 : v > 7 ? 7 : v;
+  }();
+  return w;
+}
+
 flb_pub* make_pub(const Limbs& n_in) {
   auto* K = new flb_pub();
   K->nbits = (uint32_t)H::bits(n_in);
@@ -52,7 +63,7 @@ flb_pub* make_pub(const Limbs& n_in) {
   K->n2 = H::resized(H::mul(K->n, K->n), K->s);
   H::MontCtx C(K->n2);
   K->n2_n0inv = C.n0inv;
-  K->enc = H::best_schedule(K->n, 7);
+  K->enc = H::best_schedule(K->n, sched_wmax());
   K->o_n2 = K->blob.put(K->n2, K->s);
   K->o_n = K->blob.put(K->n, K->sp);
   K->o_R2 = K->blob.put(C.R2, K->s);
@@ -101,7 +112,7 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
     R.P_n0inv = C1.n0inv;
     Limbs pm1 = P;
     H::sub_in(pm1, one);
-    R.sched = H::best_schedule(pm1, 7);
+    R.sched = H::best_schedule(pm1, sched_wmax());
     // h_P = (-Q)^-1 mod P
     Limbs negQ = P;
     H::sub_in(negQ, H::mod(Q, P));
@@ -143,8 +154,8 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
         V->half[i].o_R2 = V->blob.put(C.R2, Hf);
         V->half[i].o_R3 = V->blob.put(H::mont(C.R2, C.R2, P, C.n0inv), Hf);
       }
-      V->sched_p = H::best_schedule(V->p, 7);
-      V->sched_q = H::best_schedule(V->q, 7);
+      V->sched_p = H::best_schedule(V->p, sched_wmax());
+      V->sched_q = H::best_schedule(V->q, sched_wmax());
       V->o_sched_p = V->blob.put_raw(V->sched_p.ops);
       V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
     }

@@ -58,7 +58,8 @@ struct Cfg {
   // work row (t_hi, then the product u): 4 padding words after every 32, so the lanes of one element
   // (16 limbs = 64 bytes each, a quarter of t 128 bytes apart) hit different bank groups; rows
   // WROW words apart with WROW / 4 odd, so 8 consecutive elements do too
-  static constexpr int WPAD = S + 4 * (S / 32);
+  // (S <= 64: unpadded — two CTAs per SM must fit in the SM's 228 KB of shared memory)
+  static constexpr int WPAD = S >= 128 ? S + 4 * (S / 32) : S;
   static constexpr int WROW = (WPAD / 4) % 2 == 1 ? WPAD : WPAD + 4;
   static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB) (S = 128: all 512 columns)
   static constexpr int CTAS_PER_SM = S >= 128 ? 1 : 2;  // TMEM and shared memory per tile
@@ -70,6 +71,7 @@ struct Cfg {
   static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, NG x uint4 per element
   static constexpr int SMEM = OFF_X + kTileM * NG * 16;
   static_assert(SMEM <= 227 * 1024, "shared memory per CTA");
+  static_assert(CTAS_PER_SM * (SMEM + 1024 + 64) <= 228 * 1024, "CTAS_PER_SM tiles per SM (1 KB reserved per CTA)");
   static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
 };
 
@@ -80,8 +82,9 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)_
 __host__ __device__ __forceinline__ uint32_t cm_off(uint32_t row, uint32_t k, uint32_t kch) {
   return (row >> 3) * (kch * 128u) + (k >> 4) * 128u + (row & 7u) * 16u + (k & 15u);
 }
-// padded position of word w of a work row (4 padding words after every 32; Cfg::WROW)
-__host__ __device__ __forceinline__ int wpad(int w) { return w + 4 * (w >> 5); }
+// padded position of word w of a work row (S = 128: 4 padding words after every 32; Cfg::WPAD)
+template <int S>
+__host__ __device__ __forceinline__ int wpad(int w) { return S >= 128 ? w + 4 * (w >> 5) : w; }
 
 __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr, uint32_t sbo) {
   uint64_t d = (uint64_t)((saddr & 0x3FFFFu) >> 4);
@@ -326,7 +329,7 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
   using C = Cfg<S>;
   const int k = threadIdx.x % C::T;
   if (s.row) {
-    const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + wpad(k * C::X));
+    const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + wpad<S>(k * C::X));
 #pragma unroll
     for (int v = 0; v < C::X / 4; v++) {
       const uint4 u = q[v];
@@ -529,11 +532,11 @@ __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, i
   using C = Cfg<S>;
   if constexpr (S >= 128) {
     uint8_t* const a = sA + cm_off((uint32_t)elem, 0u, C::KCH) + 32u * (uint32_t)w;
-    uint8_t* const b = reinterpret_cast<uint8_t*>(sW + elem * C::WROW + wpad(w - S));
+    uint8_t* const b = reinterpret_cast<uint8_t*>(sW + elem * C::WROW + wpad<S>(w - S));
     return reinterpret_cast<uint4*>(w < S ? a : b);
   } else {  // (measured: the select-free form below issues fewer instructions at S <= 64)
     return w < S ? reinterpret_cast<uint4*>(sA + cm_off(elem, 4u * w, C::KCH))
-                 : reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad(w - S));
+                 : reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad<S>(w - S));
   }
 }
 
@@ -672,10 +675,10 @@ __device__ __forceinline__ void tc_square_product_w(const uint32_t (&a)[Cfg<S>::
 #pragma unroll
   for (int d = 1; d < HT; d++) {
     uint32_t v[2 * X];
-    blk_prod<X, X, T>(v, a, a, (k + d) & (T - 1), false);
     const bool wrap = k + d >= T;
     const int w0 = X * (wrap ? 2 * k + d - T : 2 * k + d);
     uint32_t c = 0;
+    blk_prod<X, X, T>(v, a, a, (k + d) & (T - 1), false);
     __syncwarp();
     if (!wrap) c = t_add_dbl<S, 2 * X>(sA, sW, elem, w0, v);
     __syncwarp();
@@ -849,7 +852,7 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
     for (int v = 0; v < X / 4; v++) {
       *reinterpret_cast<uint4*>(sA + cm_off(elem, 16u * (k * X / 4 + v), KCH)) =
           make_uint4(lo[4 * v], lo[4 * v + 1], lo[4 * v + 2], lo[4 * v + 3]);
-      *reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad(k * X + 4 * v)) =
+      *reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad<S>(k * X + 4 * v)) =
           make_uint4(hi[4 * v], hi[4 * v + 1], hi[4 * v + 2], hi[4 * v + 3]);
     }
   }
@@ -1009,8 +1012,8 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
         for (int j = 0; j < 8; j++) cv[24 + j] = g < NG - 1 ? t8[j] : top[j];
       }
       tmem_wait();
-      const uint4 h0 = reinterpret_cast<const uint4*>(row + wpad(g * QW + c0 / 4))[0];  // 8 words, one 32-block
-      const uint4 h1 = reinterpret_cast<const uint4*>(row + wpad(g * QW + c0 / 4))[1];
+      const uint4 h0 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[0];  // 8 words, one 32-block
+      const uint4 h1 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[1];
       const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
       norm8_chain<true>(cv, th, v + c0 / 4, ns, c0 == 0);
     }
@@ -1056,7 +1059,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     }
 #pragma unroll
     for (int c = 0; c < QW / 4; c++)
-      *reinterpret_cast<uint4*>(row + wpad(g * QW + 4 * c)) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+      *reinterpret_cast<uint4*>(row + wpad<S>(g * QW + 4 * c)) = make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
   }
   tc_before_sync();
   pair_sync<S>();  // the pair's rows are final (the next product / row op of these elements is the pair's)
@@ -1076,7 +1079,7 @@ __device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint
   for (int h = 0; h < C::NP; h++) {
     const int elem = prod_elem<S>(h);
     if ((uint32_t)elem < valid) {
-      const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + wpad(k * C::X));
+      const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + wpad<S>(k * C::X));
       uint4* o = reinterpret_cast<uint4*>(dst + (size_t)elem * stride + k * C::X);
 #pragma unroll
       for (int v = 0; v < C::X / 4; v++) o[v] = q[v];
@@ -1099,7 +1102,7 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
     load_const<X, C::T>(nn, Nmod);
     grp_add_small<X, C::T>(r, 1u);
     grp_cond_sub<X, C::T>(r, nn, 0u);
-    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad(k * X));
+    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad<S>(k * X));
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
@@ -1122,7 +1125,7 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
     load_const<X, C::T>(nn, Nmod);
     const uint32_t cy = grp_add<X, C::T>(r, r, a);
     grp_cond_sub<X, C::T>(r, nn, cy);
-    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad(k * X));
+    uint4* o = reinterpret_cast<uint4*>(sW + elem * C::WROW + wpad<S>(k * X));
 #pragma unroll
     for (int v = 0; v < X / 4; v++) o[v] = make_uint4(r[4 * v], r[4 * v + 1], r[4 * v + 2], r[4 * v + 3]);
   }
@@ -1371,7 +1374,7 @@ __global__ void __launch_bounds__(Cfg<S>::THREADS, 1) k_tc_debug_product(const u
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < count * 2 * S; i += C::THREADS) {
     const uint32_t e = i / (2 * S), w = i % (2 * S);
-    t[i] = w < (uint32_t)S ? *reinterpret_cast<const uint32_t*>(sA + cm_off(e, 4u * w, C::KCH)) : sW[e * C::WROW + wpad((int)w - S)];
+    t[i] = w < (uint32_t)S ? *reinterpret_cast<const uint32_t*>(sA + cm_off(e, 4u * w, C::KCH)) : sW[e * C::WROW + wpad<S>((int)w - S)];
   }
 }
 
