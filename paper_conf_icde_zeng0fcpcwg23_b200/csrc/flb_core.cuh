@@ -587,7 +587,8 @@ int launch_tc_exp_dag(flb::tc::ExpArgs& A1, flb::tc::ExpArgs& A2, cudaStream_t s
   A1.scratch = A2.scratch = (uint32_t*)s_tab.p;
   A1.tab_entries = tab1 + 1;
   A2.tab_entries = tab2 + 1;
-  flb::tc::k_tc_exp_dag<S1, S2><<<grid, flb::tc::kThreads, SMEM, st>>>(A1, A2, (uint32_t*)s_sync.p, stride);
+  static_assert(flb::tc::Cfg<S1>::THREADS == flb::tc::Cfg<S2>::THREADS, "one CTA shape for both stages");
+  flb::tc::k_tc_exp_dag<S1, S2><<<grid, flb::tc::Cfg<S2>::THREADS, SMEM, st>>>(A1, A2, (uint32_t*)s_sync.p, stride);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
 }

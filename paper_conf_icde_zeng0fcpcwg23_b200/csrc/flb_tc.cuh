@@ -44,7 +44,7 @@ struct Cfg {
   static constexpr int T = S >= 128 ? 8 : S >= 64 ? kT : 2;  // lanes per element in the product phase
   static constexpr int X = S / T;                  // limbs per lane (16)
   // threads per CTA: 8 warps (two CTAs per SM); at S = 128 (one CTA per SM: all TMEM) 16 warps, so
-  // the product phase keeps four warps per scheduler; the normalisation uses the first 8
+  // the product phase keeps four warps per scheduler
   static constexpr int THREADS = S >= 128 ? 512 : kThreads;
   static constexpr int GW = THREADS / 128;         // warps per TMEM lane quadrant
   static constexpr int EP = THREADS / T;           // elements per product pass
@@ -68,8 +68,8 @@ struct Cfg {
   static constexpr int OFF_E2 = OFF_E1 + 2 * KB * 32;       // 3 KB rows x 32 bytes
   static constexpr int OFF_A = OFF_E2 + 3 * KB * 32;        // 128 x KB bytes (core matrices)
   static constexpr int OFF_W = OFF_A + kTileM * KB;         // 128 work rows
-  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, NG x uint4 per element
-  static constexpr int SMEM = OFF_X + kTileM * NG * 16;
+  static constexpr int OFF_X = OFF_W + kTileM * WROW * 4;   // carry exchange, NG x uint2 per element
+  static constexpr int SMEM = OFF_X + kTileM * NG * 8;
   static_assert(SMEM <= 227 * 1024, "shared memory per CTA");
   static_assert(CTAS_PER_SM * (SMEM + 1024 + 64) <= 228 * 1024, "CTAS_PER_SM tiles per SM (1 KB reserved per CTA)");
   static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
@@ -887,7 +887,9 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   const bool nw = true;  // every warp normalises: column group g of elements [32 L, 32 L + 32)
   const uint32_t lane_base = sm.tmem + ((uint32_t)(32 * L) << 16);
   uint32_t* row = sW + i * C::WROW;
-  uint4* xch = reinterpret_cast<uint4*>(sm.base + C::OFF_X) + i * C::NG;
+  // carry exchange per (element, column group): x = carry (< 2^21) | all-ones flag << 29 | borrow,
+  // zero flags << 30, y = the group's word 0
+  uint2* xch = reinterpret_cast<uint2*>(sm.base + C::OFF_X) + i * C::NG;
   constexpr int NG = C::NG;
   uint2 ttop = make_uint2(0, 0);
   if (g == 0) ttop = *reinterpret_cast<const uint2*>(sA + cm_off(i, KB - 8, KCH));  // t_lo bytes KB-8 ..
@@ -906,13 +908,13 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     uint32_t ao = 0xffffffffu;
 #pragma unroll
     for (int w = 1; w < QW; w++) ao &= v[w];
-    xch[g] = make_uint4((uint32_t)carry, v[0], ao == 0xffffffffu ? 1u : 0u, 0u);
+    xch[g] = make_uint2((uint32_t)carry | (ao == 0xffffffffu ? 1u << 29 : 0u), v[0]);
   };
   // carry into half 1 (= out of half 0), and out of half 1
   auto carry_out = [&](int h, uint64_t cin) {
-    const uint4 x = xch[h];
-    const uint64_t ov = (x.z != 0u && (((uint64_t)x.y + cin) >> 32) != 0) ? 1u : 0u;
-    return (uint64_t)x.x + ov;
+    const uint2 x = xch[h];
+    const uint64_t ov = ((x.x >> 29) & 1u) != 0u && (((uint64_t)x.y + cin) >> 32) != 0 ? 1u : 0u;
+    return (uint64_t)(x.x & 0x1fffffffu) + ov;
   };
   // carry into column group gg (the prefix over the groups below it)
   auto carry_into = [&](int gg) {
@@ -1040,7 +1042,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
     br = subc_end(0u, 0u) & 1u;
 #pragma unroll
     for (int w = 0; w < QW; w++) nzd |= d[w];
-    xch[g].w = br | (nzd == 0u ? 2u : 0u);
+    xch[g].x |= (br | (nzd == 0u ? 2u : 0u)) << 30;  // (the pair reads only bits < 30 concurrently)
   }
   pair_sync<S>();
   if (nw) {
@@ -1049,7 +1051,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
 #pragma unroll
     for (int h = 0; h < NG; h++) {
       if (h == g) bin = bout;
-      const uint32_t f = xch[h].w;
+      const uint32_t f = xch[h].x >> 30;
       bout = (f & 1u) | ((f >> 1) & bout);
     }
     if (ovf != 0 || bout == 0) {                           // u >= N: take u - N
@@ -1305,7 +1307,7 @@ __global__ void __launch_bounds__(Cfg<S>::THREADS, Cfg<S>::CTAS_PER_SM) k_tc_exp
 // GPU and the end-of-launch tail is at most one stage-2 tile per CTA slot.
 // sync: [0] the tile counter, [1 + j] the flag of stage-1 tile j (zeroed before the launch).
 template <int S1, int S2>
-__global__ void __launch_bounds__(kThreads, 2) k_tc_exp_dag(const ExpArgs A1, const ExpArgs A2, uint32_t* sync,
+__global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArgs A1, const ExpArgs A2, uint32_t* sync,
                                                            uint64_t tab_stride) {
   constexpr int COLS = Cfg<S1>::TMEM_COLS > Cfg<S2>::TMEM_COLS ? Cfg<S1>::TMEM_COLS : Cfg<S2>::TMEM_COLS;
   extern __shared__ __align__(1024) uint8_t smem[];
