@@ -308,7 +308,7 @@ int flb_debug_mont_mul(const flb_pub* pub, const uint32_t* a, const uint32_t* b,
 
 /* Debug: the plain product phase of the tensor-core Montgomery kernel (csrc/flb_tc.cuh): t_i = a_i b_i
  * (square != 0: a_i^2, b ignored but must be valid) as 2 words-limb integers, for count <= 128
- * elements of words in {32, 64} limbs.  a, b: [count][words], t: [count][2 words], device.
+ * elements of words in {32, 64, 96, 128} limbs.  a, b: [count][words], t: [count][2 words], device.
  * Errors: FLB_EINVAL. */
 int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint32_t count, uint32_t words,
                          int square, void* stream);

@@ -589,7 +589,7 @@ def op_cost(key, op: str) -> Tuple[int, int]:
 
 def debug_tc_product(a: torch.Tensor, b: torch.Tensor, square: bool = False, stream=None) -> torch.Tensor:
     """The tensor-core Montgomery kernel's product phase alone: a_i b_i (or a_i^2) as 2w-limb rows,
-    w = a.shape[1] in {32, 64}, at most 128 rows (debugging and parity tests).  square: 0/False =
+    w = a.shape[1] in {32, 64, 96, 128}, at most 128 rows (debugging and parity tests).  square: 0/False =
     general product, 1/True = block squaring (one triangular diagonal square per lane), 2 = block
     squaring with the half-split diagonal square."""
     M = _check_batch(a, a.shape[1], "a")

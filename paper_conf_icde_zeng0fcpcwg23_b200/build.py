@@ -55,7 +55,7 @@ def jobs(extra):
                 obj = os.path.join(OBJ, f"flb_inst_{x}x{t}.o")
                 defs = [f"-DFLB_INST_X={x}", f"-DFLB_INST_T={t}", f"-DFLB_INST_ENC={e}", f"-DFLB_INST_DEC={d}"]
                 out.append((obj, defs + ["-c", src]))
-            for s in (32, 64, 128):
+            for s in (32, 64, 96, 128):
                 out.append((os.path.join(OBJ, f"flb_inst_tc{s}.o"), [f"-DFLB_INST_TC={s}", "-DFLB_INST_ENC=0",
                                                                       "-DFLB_INST_DEC=0", "-c", src]))
         else:

@@ -160,14 +160,15 @@ flb_priv* make_priv(const Limbs& p_in, const Limbs& q_in) {
       V->o_sched_q = V->blob.put_raw(V->sched_q.ops);
     }
   }
-  // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 moduli when sp is 32, 64 or 128
+  // tensor-core Montgomery operands (flb_tc.cuh) for the P^2 moduli when sp is 32, 64, 96 or 128
   // (decryption, key-holder encryption stage 2) and for the half-frame P moduli when H is 32 or 64
   // (key-holder encryption stage 1)
   {
     auto operands = [&](const Limbs& N, uint32_t S, size_t* e1, size_t* e2) { tc_operands(V->blob, N, S, e1, e2); };
     // (k_tc_exp starts from a table entry and needs at least one more schedule op: toy keys with
     // one-window exponents stay on the CIOS kernels)
-    if ((sp == 32 || sp == 64 || sp == 128) && V->pr[0].sched.ops.size() >= 2 && V->pr[1].sched.ops.size() >= 2) {
+    if ((sp == 32 || sp == 64 || sp == 96 || sp == 128) && V->pr[0].sched.ops.size() >= 2 &&
+        V->pr[1].sched.ops.size() >= 2) {
       for (int i = 0; i < 2; i++) operands(V->pr[i].P2, sp, &V->pr[i].o_tcE1, &V->pr[i].o_tcE2);
       V->tc = true;
     }
@@ -551,6 +552,7 @@ int flb_decrypt(const flb_priv* V, const uint32_t* c, uint32_t* m, size_t count,
   }
   if (use_tc(V)) {
     if (V->pub->sp == 128) return run_decrypt_tc<128>(V, dev, c, m, count, (cudaStream_t)stream);
+    if (V->pub->sp == 96) return run_decrypt_tc<96>(V, dev, c, m, count, (cudaStream_t)stream);
     if (V->pub->sp == 64) return run_decrypt_tc<64>(V, dev, c, m, count, (cudaStream_t)stream);
     return run_decrypt_tc<32>(V, dev, c, m, count, (cudaStream_t)stream);
   }
@@ -593,9 +595,10 @@ int flb_debug_tc_product(const uint32_t* a, const uint32_t* b, uint32_t* t, uint
                          void* stream) {
   if (!a || !b || !t || count > (uint32_t)flb::tc::kTileM) return fail(FLB_EINVAL, "null pointer or count > 128");
   if (words == 128) return run_tc_debug_product<128>(a, b, t, count, square, (cudaStream_t)stream);
+  if (words == 96) return run_tc_debug_product<96>(a, b, t, count, square, (cudaStream_t)stream);
   if (words == 64) return run_tc_debug_product<64>(a, b, t, count, square, (cudaStream_t)stream);
   if (words == 32) return run_tc_debug_product<32>(a, b, t, count, square, (cudaStream_t)stream);
-  return fail(FLB_EINVAL, "words must be 32, 64 or 128");
+  return fail(FLB_EINVAL, "words must be 32, 64, 96 or 128");
 }
 
 int flb_debug_mont_mul(const flb_pub* K, const uint32_t* a, const uint32_t* b, uint32_t* out, size_t count,
@@ -881,6 +884,7 @@ static int encrypt_crt_v2(const flb_priv* V, const uint32_t* dev, const uint32_t
   if (rc) return rc;
   if (use_tc(V)) {
     if (V->pub->sp == 128) return run_encrypt_crt_tc<128>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
+    if (V->pub->sp == 96) return run_encrypt_crt_tc<96>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
     if (V->pub->sp == 64) return run_encrypt_crt_tc<64>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
     return run_encrypt_crt_tc<32>(V, dev, m, (const uint32_t*)ys.p, c, count, st);
   }

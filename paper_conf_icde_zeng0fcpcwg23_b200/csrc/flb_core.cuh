@@ -129,7 +129,7 @@ struct flb_priv {
     // tensor-core Montgomery operands for P^2 (flb_tc.cuh): extended Toeplitz K-slices of N', N
     size_t o_tcE1 = 0, o_tcE2 = 0;
   } pr[2];
-  bool tc = false;       // P^2 tensor-core operands present (sp in {32, 64})
+  bool tc = false;       // P^2 tensor-core operands present (sp in {32, 64, 96, 128})
   bool tc_half = false;  // half-frame P tensor-core operands present (H in {32, 64})
   size_t o_one = 0;      // the integer 1
   size_t o_n = 0, o_qR_n = 0, o_qinvR_p = 0;
@@ -648,7 +648,7 @@ void tc_stage2_args(const flb_priv* V, const uint32_t* dev, const uint32_t* m, c
 template <int S>
 int tc_combine(const flb_priv* V, const uint32_t* dev, const uint32_t* cpq, uint32_t* c, size_t count,
                cudaStream_t st) {
-  constexpr int XC = 16, TC = S / 16;
+  constexpr int XC = S % 96 == 0 ? 12 : 16, TC = S / XC;  // (S = 96: eight lanes of 12 limbs)
   int cgrid;
   int rc = grid_for<TC>(flb::k_crt_combine<XC, TC>, count, &cgrid);
   if (rc) return rc;
@@ -836,7 +836,7 @@ int run_decrypt_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* c, ui
   }
   rc = launch_tc_exp<S>(A, st);
   if (rc) return rc;
-  constexpr int XF = 16, TF = S / 16;
+  constexpr int XF = S % 96 == 0 ? 12 : 16, TF = S / XF;
   int grid;
   rc = grid_for<TF>(flb::k_dec_finish<XF, TF>, count, &grid);
   if (rc) return rc;
@@ -1037,6 +1037,7 @@ FLB_ENC_COMBOS(FLB_EXTERN_ENC)
 FLB_DEC_COMBOS(FLB_EXTERN_DEC)
 FLB_TC_DECLS(extern, 32)
 FLB_TC_DECLS(extern, 64)
+FLB_TC_DECLS(extern, 96)
 FLB_TC_DECLS(extern, 128)
 FLB_TC_DAG_DECLS(extern)
 #undef FLB_EXTERN_ENC

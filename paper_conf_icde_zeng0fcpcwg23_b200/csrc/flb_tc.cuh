@@ -41,11 +41,12 @@ constexpr int kT = 4;           // lanes per element in the product phase at S =
 
 template <int S>
 struct Cfg {
-  static constexpr int T = S >= 128 ? 8 : S >= 64 ? kT : 2;  // lanes per element in the product phase
-  static constexpr int X = S / T;                  // limbs per lane (16)
+  // lanes per element in the product phase (S = 96, 3072-bit p^2: eight lanes of X = 12 limbs)
+  static constexpr int T = S >= 96 ? 8 : S >= 64 ? kT : 2;
+  static constexpr int X = S / T;                  // limbs per lane (16; 12 at S = 96)
   // threads per CTA: 8 warps (two CTAs per SM); at S = 128 (one CTA per SM: all TMEM) 16 warps, so
   // the product phase keeps four warps per scheduler
-  static constexpr int THREADS = S >= 128 ? 512 : kThreads;
+  static constexpr int THREADS = S >= 96 ? 512 : kThreads;
   static constexpr int GW = THREADS / 128;         // warps per TMEM lane quadrant
   static constexpr int EP = THREADS / T;           // elements per product pass
   static constexpr int NP = kTileM / EP;           // product passes per tile
@@ -61,8 +62,9 @@ struct Cfg {
   // (S <= 64: unpadded — two CTAs per SM must fit in the SM's 228 KB of shared memory)
   static constexpr int WPAD = S >= 128 ? S + 4 * (S / 32) : S;
   static constexpr int WROW = (WPAD / 4) % 2 == 1 ? WPAD : WPAD + 4;
-  static constexpr int TMEM_COLS = KB;             // D1 and D2 share [0, KB) (S = 128: all 512 columns)
-  static constexpr int CTAS_PER_SM = S >= 128 ? 1 : 2;  // TMEM and shared memory per tile
+  // D1 and D2 share TMEM columns [0, KB); the allocation is a power of two (S = 96, 128: all 512)
+  static constexpr int TMEM_COLS = KB <= 128 ? 128 : KB <= 256 ? 256 : 512;
+  static constexpr int CTAS_PER_SM = S >= 96 ? 1 : 2;  // TMEM and shared memory per tile
   // dynamic shared memory carve-up (bytes)
   static constexpr int OFF_E1 = 0;                          // 2 KB rows x 32 bytes
   static constexpr int OFF_E2 = OFF_E1 + 2 * KB * 32;       // 3 KB rows x 32 bytes
@@ -72,7 +74,7 @@ struct Cfg {
   static constexpr int SMEM = OFF_X + kTileM * NG * 8;
   static_assert(SMEM <= 227 * 1024, "shared memory per CTA");
   static_assert(CTAS_PER_SM * (SMEM + 1024 + 64) <= 228 * 1024, "CTAS_PER_SM tiles per SM (1 KB reserved per CTA)");
-  static_assert(X % 4 == 0 && QW % 8 == 0, "16-byte limb chunks");
+  static_assert(X % 4 == 0 && QW % 8 == 0 && KB <= 512, "16-byte limb chunks, TMEM columns");
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -540,28 +542,53 @@ __device__ __forceinline__ uint4* t_chunk(uint8_t* sA, uint32_t* sW, int elem, i
   }
 }
 
+// address of t's word w (any w) for element elem (8-byte aligned for even w)
+template <int S>
+__device__ __forceinline__ uint32_t* t_word(uint8_t* sA, uint32_t* sW, int elem, int w) {
+  using C = Cfg<S>;
+  return w < S ? reinterpret_cast<uint32_t*>(sA + cm_off((uint32_t)elem, 4u * (uint32_t)w, C::KCH))
+               : sW + elem * C::WROW + wpad<S>(w - S);
+}
+
 // t[w0 .. w0 + NW) += 2 v (mod 2^(32 NW)); returns the carry out of the region (0..2).  One carry
 // chain (add.cc / addc.cc, one IADD3.X per word) across the chunks; the doubling is a funnel shift.
-template <int S, int NW, bool DBL = true>
+// HEAD = w0 % 4 (0 or 2): a region that starts or ends half-way into a 16-byte chunk (X = 12 limbs per
+// lane at S = 96) takes a uint2 at that end.
+template <int S, int NW, bool DBL = true, int HEAD = 0>
 __device__ __forceinline__ uint32_t t_add_dbl(uint8_t* sA, uint32_t* sW, int elem, int w0, const uint32_t (&v)[NW]) {
+  static_assert((HEAD == 0 || HEAD == 2) && (NW - HEAD) % 2 == 0, "whole 8-byte pieces");
+  constexpr int NC = (NW - HEAD) / 4, TAIL = (NW - HEAD) % 4;
   uint32_t prev = 0, cy;
+  auto add = [&](uint32_t m, int i) {
+    const uint32_t x = v[i];
+    const uint32_t d = DBL ? __funnelshift_l(prev, x, 1) : x;  // (x << 1) | (prev >> 31)
+    prev = x;
+    uint32_t r;
+    if (i == 0)
+      asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(m), "r"(d));
+    else
+      asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(r) : "r"(m), "r"(d));
+    return r;
+  };
+  if constexpr (HEAD == 2) {
+    uint2* p = reinterpret_cast<uint2*>(t_word<S>(sA, sW, elem, w0));
+    const uint2 m = *p;
+    const uint32_t r0 = add(m.x, 0), r1 = add(m.y, 1);
+    *p = make_uint2(r0, r1);
+  }
 #pragma unroll
-  for (int c = 0; c < NW / 4; c++) {
-    uint4* p = t_chunk<S>(sA, sW, elem, w0 + 4 * c);
+  for (int c = 0; c < NC; c++) {
+    uint4* p = t_chunk<S>(sA, sW, elem, w0 + HEAD + 4 * c);
     const uint4 m = *p;
-    const uint32_t mm[4] = {m.x, m.y, m.z, m.w};
-    uint32_t r[4];
-#pragma unroll
-    for (int u = 0; u < 4; u++) {
-      const uint32_t x = v[4 * c + u];
-      const uint32_t d = DBL ? __funnelshift_l(prev, x, 1) : x;  // (x << 1) | (prev >> 31)
-      prev = x;
-      if (c == 0 && u == 0)
-        asm volatile("add.cc.u32 %0, %1, %2;" : "=r"(r[u]) : "r"(mm[u]), "r"(d));
-      else
-        asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(r[u]) : "r"(mm[u]), "r"(d));
-    }
-    *p = make_uint4(r[0], r[1], r[2], r[3]);
+    const uint32_t r0 = add(m.x, HEAD + 4 * c), r1 = add(m.y, HEAD + 4 * c + 1);
+    const uint32_t r2 = add(m.z, HEAD + 4 * c + 2), r3 = add(m.w, HEAD + 4 * c + 3);
+    *p = make_uint4(r0, r1, r2, r3);
+  }
+  if constexpr (TAIL == 2) {
+    uint2* p = reinterpret_cast<uint2*>(t_word<S>(sA, sW, elem, w0 + NW - 2));
+    const uint2 m = *p;
+    const uint32_t r0 = add(m.x, NW - 2), r1 = add(m.y, NW - 1);
+    *p = make_uint2(r0, r1);
   }
   asm volatile("addc.u32 %0, 0, 0;" : "=r"(cy));
   return cy + (DBL ? prev >> 31 : 0u);
@@ -697,7 +724,7 @@ __device__ __forceinline__ void tc_square_product_w(const uint32_t (&a)[Cfg<S>::
     __syncwarp();
     if (hh == 0) c = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);
     __syncwarp();
-    if (hh == 1) c = t_add_dbl<S, X + H>(sA, sW, elem, w0, v);
+    if (hh == 1) c = t_add_dbl<S, X + H, true, H % 4>(sA, sW, elem, w0, v);  // (X = 12: w0 = 2 mod 4)
     __syncwarp();
     cw[HT - 1] = c;
   }

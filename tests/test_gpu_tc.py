@@ -174,7 +174,7 @@ def test_tc_multi_tile_per_cta_both_problems():
     assert torch.equal(tc_d, m2)
 
 
-@pytest.mark.parametrize("words", [32, 64, 128])
+@pytest.mark.parametrize("words", [32, 64, 96, 128])
 @pytest.mark.parametrize("square", [0, 1, 2], ids=["general", "sqr_tri", "sqr_split"])
 def test_tc_product_phase_exact(words, square):
     """The tensor-core kernel's CUDA-core product phase (general row scan, or the block squaring
@@ -192,7 +192,7 @@ def test_tc_product_phase_exact(words, square):
         assert t[i] == want, (i, hex(t[i] ^ want))
 
 
-@pytest.mark.parametrize("words", [32, 64, 128])
+@pytest.mark.parametrize("words", [32, 64, 96, 128])
 @pytest.mark.parametrize("sq", [1, 2], ids=["tri", "split"])
 def test_tc_square_block_carries(words, sq):
     """Block squaring with triangular diagonal blocks (sqr_local: sum_{i<j} a_i a_j by lo/hi row
@@ -200,8 +200,10 @@ def test_tc_square_block_carries(words, sq):
     alternate 0xffffffff / 1 limbs, so every row chain, the doubling's shifted-out bits and the
     quarter carries hit their extremes; exact 2w-limb a^2.  sq = 2: the half-split diagonal square
     (two X/2 triangles + the doubled L H block rippled to the top), the form decryption and stage 1
-    of the key-holder encryption use."""
-    X, nb = 16, words // 16
+    of the key-holder encryption use.  S = 96: eight lanes of 12 limbs (the half block starts half-way
+    into a 16-byte chunk)."""
+    X = 12 if words == 96 else 16
+    nb = words // X
     full = (1 << (32 * X)) - 1
     alt = sum((0xFFFFFFFF if j % 2 == 0 else 1) << (32 * j) for j in range(X))
     alt2 = sum((1 if j % 2 == 0 else 0xFFFFFFFF) << (32 * j) for j in range(X))

@@ -75,15 +75,16 @@ def test_public_encrypt_tc_caller_r_edge(key):
         assert tc[i] == paillier.encrypt(n, ms[i], rs[i]), i
 
 
-@pytest.fixture(scope="module")
-def k4096():
-    p, q = KEYS["4096"]
+@pytest.fixture(scope="module", params=["3072", "4096"])
+def k4096(request):
+    p, q = KEYS[request.param]
     return flb.key_from_primes(p, q) + (p, q)
 
 
 @pytest.mark.parametrize("count", [1, 130])
 def test_decrypt_4096_tc_matches_cios_and_oracle(k4096, count):
-    """4096-bit decryption: c^(P-1) mod P^2 with P^2 of 128 words on the S = 128 kernel."""
+    """3072/4096-bit decryption: c^(P-1) mod P^2 with P^2 of 96 / 128 words on the S = 96 / 128 kernel
+    (S = 96: eight lanes of 12 limbs, KB = 384 byte columns in a 256 + 128-column MMA pair)."""
     pub, priv, p, q = k4096
     n = p * q
     m_int = synthetic.uniform_below(n, count, 1300 + count)
@@ -99,8 +100,8 @@ def test_decrypt_4096_tc_matches_cios_and_oracle(k4096, count):
 
 @pytest.mark.parametrize("count", [1, 130])
 def test_keyholder_encrypt_4096_tc_matches_cios_and_oracle(k4096, count):
-    """4096-bit key-holder encryption: stage 1 at H = 64 and stage 2 (1 + m n) y^P mod P^2 at S = 128 on
-    the tensor cores, same bits as the CIOS kernels and the oracle's Eq. 3."""
+    """3072/4096-bit key-holder encryption: stage 1 at H = 64 and stage 2 (1 + m n) y^P mod P^2 at
+    S = 96 / 128 on the tensor cores, same bits as the CIOS kernels and the oracle's Eq. 3."""
     pub, priv, p, q = k4096
     n = p * q
     m_int = synthetic.uniform_below(n, count, 1400 + count)

@@ -9,14 +9,14 @@ def timed(fn, reps=3):
         s.record(); fn(); e.record(); torch.cuda.synchronize(); ts.append(s.elapsed_time(e)/1e3)
     return statistics.median(ts)
 out={}
-for bits,count in ((2048,133160),(1024,133160),(4096,16384)):
+for bits,count in ((2048,133160),(1024,133160),(3072,16384),(4096,16384)):
     pub, priv = flb.keygen(bits, 0xF1B0+bits)
     g=torch.Generator().manual_seed(1)
     m=torch.randint(-2**31,2**31-1,(count,bits//32),generator=g,dtype=torch.int32); m[:,-1]=0; m=m.cuda()
     for tc in ("1","0"):
         os.environ["FLB_TC"]=tc
         out["%d_pub_enc_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.encrypt(pub,m,seed=3)))
-        if bits==4096:
+        if bits>=3072:
             c=flb.encrypt_crt(priv,m,seed=3)
             out["%d_dec_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.decrypt(priv,c)))
             out["%d_kh_enc_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.encrypt_crt(priv,m,seed=3)))
