@@ -258,11 +258,18 @@ __device__ __forceinline__ void norm8_chain(const uint32_t (&cv)[32], const uint
   st.hprev = hi[7];
 }
 
+// np: product passes of the current unit (Cfg::NP for a whole tile, 1 for a half unit: k_tc_exp)
 struct Smem {
   uint8_t* base;
   uint32_t tmem;
   uint64_t* mbar;
+  int np;
 };
+
+// Half units (k_tc_exp's last, incomplete round of tiles): 64 elements on the rows of product pass 0,
+// rows r with r % 32 < 16 (prod_elem); element index of row r of a half unit, relative to its first
+// element.  Whole tiles: the identity.
+__device__ __forceinline__ int unit_index(int row, bool half) { return half ? ((row >> 5) << 4) + (row & 15) : row; }
 
 // An operand of tc_mont per element of the tile: the element's work row (row = true), or element j
 // of an array at p + j * stride with `words` limbs (the rest zero; elements >= `valid` read zeros;
@@ -278,11 +285,12 @@ struct Src {
   uint32_t stride, words, valid;
   bool row;
   uint32_t ld;
+  bool half;  // rows map to the elements of a half unit (unit_index)
 };
-__device__ __forceinline__ Src src_row() { return Src{nullptr, 0, 0, 0, true, kLdNC}; }
+__device__ __forceinline__ Src src_row() { return Src{nullptr, 0, 0, 0, true, kLdNC, false}; }
 __device__ __forceinline__ Src src_arr(const uint32_t* p, uint32_t stride, uint32_t words, uint32_t valid,
-                                       uint32_t ld = kLdNC) {
-  return Src{p, stride, words, valid, false, ld};
+                                       uint32_t ld = kLdNC, bool half = false) {
+  return Src{p, stride, words, valid, false, ld, half};
 }
 
 __device__ __forceinline__ uint4 ld_v4(const uint32_t* p, uint32_t ld) {
@@ -339,9 +347,10 @@ __device__ __forceinline__ void src_load(uint32_t (&r)[Cfg<S>::X], const Src& s,
     }
   } else {
     // limbs [k X, k X + X) of the element (the rest of a short element reads zeros)
-    const uint32_t* base = s.p + (size_t)elem * s.stride;
+    const int j = unit_index(elem, s.half);
+    const uint32_t* base = s.p + (size_t)j * s.stride;
     const uint32_t w0 = (uint32_t)(k * C::X);
-    const bool valid = (uint32_t)elem < s.valid;
+    const bool valid = (uint32_t)j < s.valid;
     if (valid && w0 + C::X <= s.words) {
 #pragma unroll
       for (int v = 0; v < C::X / 4; v++) {
@@ -819,14 +828,15 @@ __device__ __forceinline__ void tc_square_product_t2(const uint32_t (&a)[Cfg<S>:
 // elements' sA rows (the MMA A operand), t_hi into their work rows.  Groups of T lanes per element
 // (X = 16 limbs each), NP passes of EP elements.  CTA-collective (no trailing barrier).
 template <int S, int SQ = FLB_TC_TRISQ>
-__device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq, uint8_t* sA, uint32_t* sW) {
+__device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq, uint8_t* sA, uint32_t* sW,
+                                           int np = Cfg<S>::NP) {
   using C = Cfg<S>;
   constexpr int X = C::X, KCH = C::KCH;
   constexpr int T = C::T;
   const int tid = threadIdx.x, k = tid % T;
-  // ---- P: t = a b, NP passes of EP elements (S = 64: two passes of 64; S = 32: one of 128)
+  // ---- P: t = a b, np passes of EP elements (S = 64: two passes of 64; S = 32: one of 128)
 #pragma unroll 1
-  for (int h = 0; h < C::NP; h++) {
+  for (int h = 0; h < np; h++) {
     const int elem = prod_elem<S>(h);
     uint32_t a[X], b[X];
     src_load<S>(a, sa, elem, sW);
@@ -898,7 +908,7 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
 #if FLB_TC_PROF
   long long t_ = clock64();
 #endif
-  tc_product<S, SQ>(sa, sb, sq, sA, sW);
+  tc_product<S, SQ>(sa, sb, sq, sA, sW, sm.np);
   fence_async_smem();
   tc_before_sync();
   __syncthreads();
@@ -1098,18 +1108,21 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
 #endif
 }
 
-// copy each element's work row (words 0..S-1) to dst + j * stride (elements j < valid)
+// copy each element's work row (words 0..S-1) to dst + j * stride (elements j < valid; j = unit_index of
+// the row when half)
 template <int S>
-__device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint32_t stride, uint32_t valid) {
+__device__ __forceinline__ void tc_row_store(const Smem& sm, uint32_t* dst, uint32_t stride, uint32_t valid,
+                                             bool half = false) {
   using C = Cfg<S>;
   const uint32_t* sW = reinterpret_cast<const uint32_t*>(sm.base + C::OFF_W);
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < C::NP; h++) {
+  for (int h = 0; h < sm.np; h++) {
     const int elem = prod_elem<S>(h);
-    if ((uint32_t)elem < valid) {
+    const int j = unit_index(elem, half);
+    if ((uint32_t)j < valid) {
       const uint4* q = reinterpret_cast<const uint4*>(sW + elem * C::WROW + wpad<S>(k * C::X));
-      uint4* o = reinterpret_cast<uint4*>(dst + (size_t)elem * stride + k * C::X);
+      uint4* o = reinterpret_cast<uint4*>(dst + (size_t)j * stride + k * C::X);
 #pragma unroll
       for (int v = 0; v < C::X / 4; v++) o[v] = q[v];
     }
@@ -1124,7 +1137,7 @@ __device__ __forceinline__ void tc_row_add_one(const Smem& sm, const uint32_t* _
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < C::NP; h++) {
+  for (int h = 0; h < sm.np; h++) {
     const int elem = prod_elem<S>(h);
     uint32_t r[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
@@ -1146,7 +1159,7 @@ __device__ __forceinline__ void tc_row_add(const Smem& sm, const Src& s, const u
   uint32_t* sW = reinterpret_cast<uint32_t*>(sm.base + C::OFF_W);
   const int k = threadIdx.x % C::T;
 #pragma unroll 1
-  for (int h = 0; h < C::NP; h++) {
+  for (int h = 0; h < sm.np; h++) {
     const int elem = prod_elem<S>(h);
     uint32_t r[X], a[X], nn[X];
     src_load<S>(r, src_row(), elem, sW);
@@ -1211,25 +1224,29 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
 
 // One tile (128 elements) of problem P: the element powers x^E (or (1 + m n) x^E) into P.out.  `tab`
 // is the CTA's window-table scratch ([entry][kTileM][S] words).  The Toeplitz operands of P are in
-// shared memory (tc_load_operands).
+// shared memory (tc_load_operands).  hf >= 0: half unit hf of the tile (its elements 64 hf .. 64 hf + 63
+// on the rows of product pass 0, sm.np = 1).
 template <int S, int SQ = FLB_TC_TRISQ>
 __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, const uint32_t* one, uint32_t* tab,
-                                            const Smem& sm, uint32_t& phase, uint32_t x_ld = kLdNC) {
+                                            const Smem& sm, uint32_t& phase, uint32_t x_ld = kLdNC, int hf = -1) {
   const Src row = src_row();
   const int TB = P.table;
+  const bool half = hf >= 0;
   auto slot = [&](int ent) { return src_arr(tab + (size_t)ent * kTileM * S, S, S, kTileM, kLdCTA); };
   auto slot_ptr = [&](int ent) { return tab + (size_t)ent * kTileM * S; };
-  const uint64_t e0 = tile * kTileM;
-  const uint32_t nvalid = (uint32_t)((P.count - e0) < (uint64_t)kTileM ? (P.count - e0) : (uint64_t)kTileM);
+  const uint64_t e0 = tile * kTileM + (half ? (uint64_t)(kTileM / 2) * hf : 0u);
+  const uint64_t cap = half ? kTileM / 2 : kTileM;
+  // (the second half unit of a last tile with <= 64 elements is empty)
+  const uint32_t nvalid = e0 >= P.count ? 0u : (uint32_t)((P.count - e0) < cap ? (P.count - e0) : cap);
   const uint32_t* xb = P.x + e0 * P.x_stride;
   if (P.x_words <= (uint32_t)S) {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid, x_ld), src_arr(P.R2, 0, S, kTileM), false, sm, P.N,
-                   phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm,
+                   P.N, phase);
   } else {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid, x_ld), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
     tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
-    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid, x_ld), src_arr(P.R3, 0, S, kTileM), false, sm, P.N,
-               phase);                                      // hi R^2
+    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid, x_ld, half), src_arr(P.R3, 0, S, kTileM), false,
+                   sm, P.N, phase);                         // hi R^2
     tc_row_add<S>(sm, slot(0), P.N);
   }
   tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
@@ -1260,14 +1277,14 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
   }
   if (P.m) {
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
-    tc_mont<S, SQ>(src_arr(P.m + e0 * P.m_stride, P.m_stride, P.m_words, nvalid), src_arr(P.nR, 0, S, kTileM), false,
-                   sm, P.N, phase);                         // m n
+    tc_mont<S, SQ>(src_arr(P.m + e0 * P.m_stride, P.m_stride, P.m_words, nvalid, kLdNC, half),
+                   src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
     tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
     tc_mont<S, SQ>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
   } else {
     tc_mont<S, SQ>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
   }
-  tc_row_store<S>(sm, P.out + e0 * S, S, nvalid);
+  tc_row_store<S>(sm, P.out + e0 * S, S, nvalid, half);
 }
 
 // CTA prologue / epilogue shared by the modexp kernels: the MMA-completion mbarrier and COLS TMEM columns
@@ -1303,12 +1320,21 @@ __global__ void __launch_bounds__(Cfg<S>::THREADS, Cfg<S>::CTAS_PER_SM) k_tc_exp
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t tmem_sh;
   tc_cta_init<C::TMEM_COLS>(&mbar, &tmem_sh);
-  const Smem sm{smem, tmem_sh, &mbar};
+  const Smem sm{smem, tmem_sh, &mbar, C::NP};
+  const Smem sm_half{smem, tmem_sh, &mbar, 1};
   uint32_t phase = 0;
   const uint64_t tiles_all = A.pb[0].tiles + (A.nprob > 1 ? A.pb[1].tiles : 0);
+  // The K tiles of an incomplete last round run as 2K half units of one product pass (≈ 0.6 of a
+  // tile's time) when that still fits one round (2K <= grid): a shorter tail.
+  const uint64_t rem = tiles_all % gridDim.x;
+  const uint64_t K = (C::NP == 2 && 2 * rem <= gridDim.x) ? rem : 0;
+  const uint64_t units = tiles_all + K;
   int loaded = -1;
   uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * A.tab_entries * S;
-  for (uint64_t gt = blockIdx.x; gt < tiles_all; gt += gridDim.x) {
+  for (uint64_t u = blockIdx.x; u < units; u += gridDim.x) {
+    const bool whole = u < tiles_all - K;
+    const uint64_t gt = whole ? u : tiles_all - K + (u - (tiles_all - K)) / 2;
+    const int hf = whole ? -1 : (int)((u - (tiles_all - K)) & 1u);
     const int pi = gt < A.pb[0].tiles ? 0 : 1;
     const ExpProblem& P = A.pb[pi];
     if (pi != loaded) {
@@ -1318,7 +1344,8 @@ __global__ void __launch_bounds__(Cfg<S>::THREADS, Cfg<S>::CTAS_PER_SM) k_tc_exp
       __syncthreads();
       loaded = pi;
     }
-    tc_exp_tile<S, FLB_TC_TRISQ_EXP>(P, pi == 0 ? gt : gt - A.pb[0].tiles, A.one, tab, sm, phase);
+    tc_exp_tile<S, FLB_TC_TRISQ_EXP>(P, pi == 0 ? gt : gt - A.pb[0].tiles, A.one, tab, whole ? sm : sm_half, phase,
+                                     kLdNC, hf);
     __syncthreads();  // the work rows are rewritten by the next tile's first product
   }
   tc_cta_fini<C::TMEM_COLS>(tmem_sh);
@@ -1341,7 +1368,7 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t tmem_sh, next;
   tc_cta_init<COLS>(&mbar, &tmem_sh);
-  const Smem sm{smem, tmem_sh, &mbar};
+  const Smem sm1{smem, tmem_sh, &mbar, Cfg<S1>::NP}, sm2{smem, tmem_sh, &mbar, Cfg<S2>::NP};
   uint32_t phase = 0;
   const uint64_t T1 = A1.pb[0].tiles + A1.pb[1].tiles, T2 = A2.pb[0].tiles + A2.pb[1].tiles;
   int loaded = -1;  // 2 * stage + prime
@@ -1374,9 +1401,9 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
         }
       }
       __syncthreads();
-      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, sm, phase, kLdGPU);  // y: written by another CTA of this launch
+      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, sm2, phase, kLdGPU);  // y: written by another CTA of this launch
     } else {
-      tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm, phase);
+      tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm1, phase);
     }
     __syncthreads();  // the tile's output rows are stored; the work rows are rewritten next
     if (threadIdx.x == 0) {

@@ -61,6 +61,23 @@ def test_public_encrypt_tc_matches_cios_and_oracle(key, count):
     assert from_dev(flb.decrypt(priv, tc)) == m_int
 
 
+@pytest.mark.parametrize("extra", [1, 64, 100, 128 * 5 + 3])
+def test_public_encrypt_tc_half_units(key, extra):
+    """Batches one round of the persistent grid plus a few tiles: the last, incomplete round runs as half
+    units (64 elements on the rows of product pass 0, one pass) — including an empty second half and a
+    ragged first half; bit-exact against CIOS."""
+    pub, priv, p, q = key
+    n = p * q
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    per_sm = 1 if pub.ct_words >= 96 else 2  # k_tc_exp CTAs per SM (flb_tc.cuh Cfg::CTAS_PER_SM)
+    count = sms * per_sm * 128 + extra
+    m = to_dev(synthetic.uniform_below(n, count, 1150 + extra), pub.pt_words)
+    tc = _env(lambda: flb.encrypt(pub, m, seed=0x4A11, ctr0=2), "1")
+    cios = _env(lambda: flb.encrypt(pub, m, seed=0x4A11, ctr0=2), "0")
+    bad = (tc != cios).any(dim=1).nonzero().flatten().tolist()
+    assert not bad, (len(bad), bad[:5])
+
+
 def test_public_encrypt_tc_caller_r_edge(key):
     """caller-supplied r: r = 1 (Enc(m; 1) = 1 + m n), r = n - 1, r = p (not a unit: the function is still
     defined as the integer formula)."""
