@@ -470,9 +470,21 @@ def run_flb(args):
     e2e = None
     if not args.no_e2e:
         import numpy as np
-        grads_np = [g.numpy() for g in grads_host]
+
+        def pinned(shape, dtype):
+            # page-locked host buffers (the host pipeline DMAs straight from / into them)
+            t = torch.empty(shape, dtype=torch.int32 if dtype == np.uint32 else torch.float32, pin_memory=True)
+            return t.numpy().view(dtype)
+
+        grads_np = []
+        for g in grads_host:
+            gp = pinned(tuple(g.shape), np.float32)
+            gp[...] = g.numpy()
+            grads_np.append(gp)
         offs_np, idx_np = offs.cpu().numpy(), idx.cpu().numpy()
-        cts_h = np.empty((CLIENTS * rows, ctw), dtype=np.uint32)
+        cts_h = pinned((CLIENTS * rows, ctw), np.uint32)
+        part_out = pinned((len(offs_np) - 1, ctw), np.uint32)
+        vals_out = pinned((max(my_values, 1),), np.float32)
         kh = priv if args.encrypt == "keyholder" else None
         h2d = d2h = 0
 
@@ -483,7 +495,7 @@ def run_flb(args):
                                         out=cts_h)
             h2d += sum(g.nbytes for g in grads_np)
             d2h += cts_h.nbytes
-            part_h = flb.reduce_segments_host(pub, cts_h, offs_np, idx_np, max_segment_len=CLIENTS)
+            part_h = flb.reduce_segments_host(pub, cts_h, offs_np, idx_np, max_segment_len=CLIENTS, out=part_out)
             h2d += cts_h.nbytes + offs_np.nbytes + idx_np.nbytes
             d2h += part_h.nbytes
             if world > 1:
@@ -495,7 +507,7 @@ def run_flb(args):
             else:
                 fin_h = part_h[:rows]
             if my_values:
-                flb.decrypt_unpack_host(priv, cd, fin_h, my_values, summands=CLIENTS * world)
+                flb.decrypt_unpack_host(priv, cd, fin_h, my_values, summands=CLIENTS * world, out=vals_out[:my_values])
                 h2d += fin_h.nbytes
                 d2h += my_values * 4
 
@@ -517,7 +529,7 @@ def run_flb(args):
             e_ms, h2d, d2h = float(tm[0]), float(t[1]), float(t[2])
         e2e = {"value": total_ops / (e_ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": e_ms,
-               "path": "C-ABI host-buffer pipeline: flb_pack_encrypt_host_multi (%d clients) -> flb_reduce_segments_host "
+               "path": "C-ABI host-buffer pipeline over page-locked host arrays: flb_pack_encrypt_host_multi (%d clients) -> flb_reduce_segments_host "
                        "-> %sflb_decrypt_unpack_host; host wall clock per step" %
                        (CLIENTS, "NCCL all_to_all + finish -> " if world > 1 else "")}
 

@@ -513,11 +513,21 @@ def pack_encrypt_host(pub: PublicKey, codec: Codec, x, seed: int = 0, ctr0: int 
     M = codec.num_plaintexts(x.shape[0])
     if out is None:
         out = np.empty((M, pub.ct_words), dtype=np.uint32)
+    _check_host_out(out, (M, pub.ct_words), np.uint32, "out")
     cs = codec.struct()
     check("flb_pack_encrypt_host", LIB.flb_pack_encrypt_host(pub.handle, priv.handle if priv else None,
                                                              ctypes.byref(cs), _np_ptr(x), x.shape[0],
                                                              seed & 0xFFFFFFFFFFFFFFFF, ctr0, _np_ptr(out)))
     return out
+
+
+def _check_host_out(out, shape, dtype, what):
+    """A caller-supplied host output: C-contiguous numpy array of exactly this shape and dtype (it may live
+    in page-locked memory, e.g. a pin_memory tensor's .numpy(): the pipeline then copies into it directly)."""
+    import numpy as np
+    if not isinstance(out, np.ndarray) or out.dtype != dtype or tuple(out.shape) != tuple(shape) \
+            or not out.flags["C_CONTIGUOUS"]:
+        raise ValueError("%s must be a C-contiguous %s array of shape %s" % (what, np.dtype(dtype).name, tuple(shape)))
 
 
 def pack_encrypt_host_multi(pub: PublicKey, codec: Codec, xs, seed: int = 0, ctr0: int = 0,
@@ -529,6 +539,7 @@ def pack_encrypt_host_multi(pub: PublicKey, codec: Codec, xs, seed: int = 0, ctr
     M = sum(codec.num_plaintexts(x.shape[0]) for x in xs)
     if out is None:
         out = np.empty((M, pub.ct_words), dtype=np.uint32)
+    _check_host_out(out, (M, pub.ct_words), np.uint32, "out")
     ptrs = (ctypes.c_void_p * len(xs))(*[x.ctypes.data for x in xs])
     lens = (ctypes.c_size_t * len(xs))(*[x.shape[0] for x in xs])
     cs = codec.struct()
@@ -543,8 +554,11 @@ def decrypt_unpack_host(priv: PrivateKey, codec: Codec, c, n_values: int, summan
     """Host ciphertexts -> host float32 values, pipelined (PAPER Fig. 4 ⑤–⑨)."""
     import numpy as np
     c = np.ascontiguousarray(c, dtype=np.uint32)
+    if c.ndim != 2 or c.shape[1] != priv.pub.ct_words or c.shape[0] < codec.num_plaintexts(n_values):
+        raise ValueError("c must be [>= %d, %d] ciphertext limbs" % (codec.num_plaintexts(n_values), priv.pub.ct_words))
     if out is None:
         out = np.empty((n_values,), dtype=np.float32)
+    _check_host_out(out, (n_values,), np.float32, "out")
     cs = codec.struct()
     if isinstance(summands, int):
         sp, ss = None, summands
@@ -566,8 +580,11 @@ def reduce_segments_host(pub: PublicKey, c, offsets, idx=None, max_segment_len: 
     if idx is not None:
         idx = np.ascontiguousarray(idx, dtype=np.int64)
         ip = _np_ptr(idx)
+    if c.ndim != 2 or c.shape[1] != pub.ct_words:
+        raise ValueError("c must be [count, %d] ciphertext limbs" % pub.ct_words)
     if out is None:
         out = np.empty((S, pub.ct_words), dtype=np.uint32)
+    _check_host_out(out, (S, pub.ct_words), np.uint32, "out")
     check("flb_reduce_segments_host", LIB.flb_reduce_segments_host(pub.handle, _np_ptr(c), c.shape[0], ip,
                                                                    _np_ptr(offsets), S, max_segment_len,
                                                                    _np_ptr(out)))

@@ -72,3 +72,43 @@ def test_multi_array_host_encrypt_equals_per_array_calls():
             parts.append(flb.pack_encrypt_host(pub, cd, x, seed=21, ctr0=ctr, priv=priv))
             ctr += cd.num_plaintexts(x.shape[0])
     assert np.array_equal(multi, np.concatenate(parts))
+
+
+def _pinned(shape, dtype):
+    t = torch.empty(shape, dtype=torch.int32 if dtype == np.uint32 else torch.float32, pin_memory=True)
+    return t.numpy().view(dtype)
+
+
+def test_host_pipeline_page_locked_buffers():
+    """Page-locked caller buffers (pin_memory tensors): the pipeline DMAs straight from / into them
+    (no staging copy) and the bits equal the pageable-buffer calls; 8 clients of 16,645 + a ragged
+    remainder, so the encryption runs as several equal chunks (flb_host_pipeline.cu chunk_rows)."""
+    p, q = golden_keys()["2048"]
+    pub, priv = flb.key_from_primes(p, q)
+    S, clients = 63, 8
+    cd = flb.Codec(1.0, 29, 3, S)
+    nv = 16645 * S - 5
+    xs = [synthetic.c2_gradient(c, n=nv) for c in range(clients)]
+    xs_p = []
+    for x in xs:
+        xp = _pinned(x.shape, np.float32)
+        xp[...] = x
+        xs_p.append(xp)
+    rows = cd.num_plaintexts(nv)
+    cts_p = _pinned((clients * rows, pub.ct_words), np.uint32)
+    flb.pack_encrypt_host_multi(pub, cd, xs_p, seed=21, priv=priv, out=cts_p)
+    cts = flb.pack_encrypt_host_multi(pub, cd, xs, seed=21, priv=priv)
+    assert np.array_equal(cts_p, cts)
+    offs, idx = fdist.client_segments(clients, rows)
+    agg_p = _pinned((rows, pub.ct_words), np.uint32)
+    flb.reduce_segments_host(pub, cts_p, offs.numpy(), idx.numpy(), max_segment_len=clients, out=agg_p)
+    agg = flb.reduce_segments_host(pub, cts, offs.numpy(), idx.numpy(), max_segment_len=clients)
+    assert np.array_equal(agg_p, agg)
+    out_p = _pinned((nv,), np.float32)
+    flb.decrypt_unpack_host(priv, cd, agg_p, nv, summands=clients, out=out_p)
+    out = flb.decrypt_unpack_host(priv, cd, agg, nv, summands=clients)
+    assert np.array_equal(out_p.view(np.uint32), out.view(np.uint32))
+    exact = np.sum(np.array(xs, dtype=np.float64), axis=0)
+    assert np.max(np.abs(out_p - exact)) <= clients / ((1 << 29) - 1) + 1e-6
+    with pytest.raises(ValueError):
+        flb.reduce_segments_host(pub, cts_p, offs.numpy(), idx.numpy(), max_segment_len=clients, out=agg_p[:-1])
