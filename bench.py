@@ -455,8 +455,13 @@ def run_flb(args):
         "reduce (hom-add products, k_reduce CIOS)": add_lp * red_units / (phase["t_red"] * 1e-3) / 1e12 / peak,
     }
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "encrypt_traffic.json" if args.encrypt == "public" else
-                      ("r02_encrypt_tc_traffic.json" if enc_tc else "encrypt_crt_traffic.json"))
+    # DRAM bytes per launch of the dominant kernel from the round's ncu --set full capture
+    # (tools/traffic_from_ncu.py)
+    if args.encrypt == "public":
+        tp = "r02_encrypt_pub_tc_traffic.json" if tc_on else "encrypt_traffic.json"
+    else:
+        tp = "r02_encrypt_tc_traffic.json" if enc_tc else "encrypt_crt_traffic.json"
+    tp = os.path.join(ROOT, "profiles", tp)
     if os.path.exists(tp):
         try:
             with open(tp) as f:
