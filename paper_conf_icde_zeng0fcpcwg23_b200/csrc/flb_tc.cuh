@@ -1369,17 +1369,26 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
   __shared__ uint32_t tmem_sh, next;
   tc_cta_init<COLS>(&mbar, &tmem_sh);
   const Smem sm1{smem, tmem_sh, &mbar, Cfg<S1>::NP}, sm2{smem, tmem_sh, &mbar, Cfg<S2>::NP};
+  const Smem sm2h{smem, tmem_sh, &mbar, 1};
   uint32_t phase = 0;
   const uint64_t T1 = A1.pb[0].tiles + A1.pb[1].tiles, T2 = A2.pb[0].tiles + A2.pb[1].tiles;
+  // the last K2 stage-2 tiles (those beyond whole rounds of the grid) run as 2 K2 half units (as in
+  // k_tc_exp): the queue holds T1 stage-1 tiles, then T2 - K2 stage-2 tiles, then 2 K2 half units
+  const uint64_t rem2 = T2 % gridDim.x;
+  const uint64_t K2 = (Cfg<S2>::NP == 2 && 2 * rem2 <= gridDim.x) ? rem2 : 0;
+  const uint64_t U2 = T2 + K2;
   int loaded = -1;  // 2 * stage + prime
   uint32_t* tab = A1.scratch + (size_t)blockIdx.x * tab_stride;
   if (threadIdx.x == 0) next = atomicAdd(sync, 1u);
   __syncthreads();
   for (;;) {
     const uint64_t gt = next;
-    if (gt >= T1 + T2) break;
+    if (gt >= T1 + U2) break;
     const bool st2 = gt >= T1;
-    const uint64_t j = st2 ? gt - T1 : gt;
+    const uint64_t u = st2 ? gt - T1 : gt;
+    const bool whole = !st2 || u < T2 - K2;
+    const uint64_t j = whole ? u : T2 - K2 + (u - (T2 - K2)) / 2;  // tile (stage 2: also its stage-1 tile)
+    const int hf = whole ? -1 : (int)((u - (T2 - K2)) & 1u);
     const ExpArgs& A = st2 ? A2 : A1;
     const int pi = j < A.pb[0].tiles ? 0 : 1;
     const ExpProblem& P = A.pb[pi];
@@ -1401,7 +1410,8 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
         }
       }
       __syncthreads();
-      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, sm2, phase, kLdGPU);  // y: written by another CTA of this launch
+      // y: written by another CTA of this launch
+      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, whole ? sm2 : sm2h, phase, kLdGPU, hf);
     } else {
       tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm1, phase);
     }

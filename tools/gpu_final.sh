@@ -22,9 +22,9 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
   -k regex:k_tc_exp_dag -c 1 -o gpurun_out/${TAG}_ncu_encrypt python tools/prof_c2.py > gpurun_out/${TAG}_ncu_encrypt.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-  -k 'regex:k_tc_exp<64>' -c 1 -o gpurun_out/${TAG}_ncu_decrypt python tools/prof_dec.py > gpurun_out/${TAG}_ncu_decrypt.log 2>&1
+  -k 'regex:k_tc_exp<.int.64>' -c 1 -o gpurun_out/${TAG}_ncu_decrypt python tools/prof_dec.py > gpurun_out/${TAG}_ncu_decrypt.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-  -k 'regex:k_tc_exp<128>' -c 1 -o gpurun_out/${TAG}_ncu_public python tools/prof_pub.py 133160 > gpurun_out/${TAG}_ncu_public.log 2>&1
+  -k 'regex:k_tc_exp<.int.128>' -c 1 -o gpurun_out/${TAG}_ncu_public python tools/prof_pub.py 133160 > gpurun_out/${TAG}_ncu_public.log 2>&1
 # (compute-sanitizer is closed on this GPU pool: the parity suites and FLB_DEBUG_CHECKS stand in)
 cat gpurun_out/${TAG}_pytest_gpu.txt gpurun_out/${TAG}_smoke.txt
 for f in gpurun_out/${TAG}_bench*.json; do echo "$f"; head -c 300 "$f"; echo; done
