@@ -407,8 +407,15 @@ def run_flb(args):
             enc_kernel = "k_crt_pre<16,2> + k_encrypt_crt2<16,4> (two-stage key-holder encryption)"
     else:
         enc_mm, enc_lp = flb.op_cost(pub, "encrypt")
-        enc_kernel = "k_encrypt<16,8>"
         enc_tc = None
+        if tc_on:
+            try:  # public-key encryption in the n^2 frame on the tensor cores (k_tc_exp<128> at 2048 bits)
+                enc_tc = flb.op_cost(pub, "encrypt_tc")
+                enc_macs = flb.op_cost(pub, "encrypt_tc_macs")[1]
+            except flb.FlbError:
+                enc_tc = None
+        enc_kernel = ("k_tc_exp<%d> (public-key encryption (1 + m n) r^n mod n^2 in the n^2 frame; Montgomery "
+                      "reduction as u8 tcgen05 MMAs, t = a b on the IMAD pipe)" % ctw) if enc_tc else "k_encrypt<16,8>"
     dec_mm, dec_lp = flb.op_cost(priv, "decrypt")
     enc_units = CLIENTS * rows
     sm_mhz_max = clk.get("sm_max_mhz") or 1965.0

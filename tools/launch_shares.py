@@ -35,10 +35,15 @@ def main():
             name += " (decryption)"
         tot[name] += ms
         cnt[name] += 1
-    step = sum(v for k, v in tot.items() if "k_encrypt<" not in k)
+    # the bench's separately timed public-key encryption (k_encrypt, or k_tc_exp<128> + its Philox fill
+    # in the n^2 frame at 2048 bits) is not part of the key-holder C2 step
+    def public(k):
+        return "k_encrypt<" in k or "k_tc_exp<128>" in k or "k_tc_exp<(int)128>" in k
+
+    step = sum(v for k, v in tot.items() if not public(k))
     out = {"source": note, "kernels": {}}
     for k, v in tot.most_common():
-        pub = "k_encrypt<" in k
+        pub = public(k)
         out["kernels"][k] = {"launches": cnt[k], "total_ms": round(v, 3),
                              "share_of_step_pct": None if pub else round(100 * v / step, 3)}
     print(json.dumps(out, indent=1))
