@@ -92,7 +92,10 @@ uint32_t flb_slot_capacity(const flb_pub* pub, uint32_t slot_bits);
  * computed as (1 + m_i n) r_i^n.  m: [count][pt_words], each m_i < n.  r: [count][pt_words]
  * caller randomness (each r_i < n, gcd(r_i, n) = 1), or NULL to draw r_i on the device from
  * Philox4x32-10 with key = seed and counter (ctr0 + i, j) exactly as oracle/philox.py draw_r
- * (reading c4).  c: [count][ct_words].  count = 0 is a no-op.  Errors: FLB_EINVAL, FLB_ECUDA. */
+ * (reading c4).  c: [count][ct_words].  count = 0 is a no-op.  For 1024/2048-bit keys (n^2 of 64/128
+ * words) a batch of at least 96 elements per SM runs on the tensor-core Montgomery kernel (see
+ * flb_encrypt_crt); smaller batches, FLB_TC=0 and larger keys run the CIOS kernel (same bits;
+ * FLB_TC=2 forces the tensor cores at any size).  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_encrypt(const flb_pub* pub, const uint32_t* m, const uint32_t* r, uint64_t seed,
                 uint64_t ctr0, uint32_t* c, size_t count, void* stream);
 
@@ -101,7 +104,7 @@ int flb_encrypt(const flb_pub* pub, const uint32_t* m, const uint32_t* r, uint64
  * recombined by CRT (c = c_q + q^2 ((c_p - c_q) (q^2)^-1 mod p^2)) — about half the limb products.
  * Beyond the paper; in Fig. 2 the clients that encrypt also
  * decrypt, so they hold the key.  From 2048 bits the exponentiation is two-stage,
- * r^n mod P^2 = (r^Q mod P)^P mod P^2; for 1024/2048-bit keys (P^2 of 32/64 words) and the
+ * r^n mod P^2 = (r^Q mod P)^P mod P^2; for 1024-4096-bit keys (P^2 of 32/64/96/128 words) and the
  * half-frame first stage at 2048-4096 bits every Montgomery product runs its reduction
  * q = t N' mod R, (t + q N)/R as u8 tcgen05 MMAs against Toeplitz matrices of N' and N (the batch
  * shares N) with TMEM accumulators (csrc/flb_tc.cuh); FLB_TC=0 in the environment selects the
@@ -112,8 +115,8 @@ int flb_encrypt_crt(const flb_priv* priv, const uint32_t* m, const uint32_t* r, 
 
 /* Paillier::decrypt (Eq. 4), by CRT (reading c10).  c: [count][ct_words]
  * (each a unit < n^2), m: [count][pt_words] receives m_i in [0, n).  For 1024/2048-bit keys the two
- * exponentiations c^(P-1) mod P^2 run on the tensor-core Montgomery kernel (see flb_encrypt_crt;
- * FLB_TC=0 selects CIOS, same bits).  Errors: FLB_EINVAL, FLB_ECUDA. */
+ * exponentiations c^(P-1) mod P^2 run on the tensor-core Montgomery kernel (3072/4096-bit keys too:
+ * P^2 of 96/128 words; see flb_encrypt_crt; FLB_TC=0 selects CIOS, same bits).  Errors: FLB_EINVAL, FLB_ECUDA. */
 int flb_decrypt(const flb_priv* priv, const uint32_t* c, uint32_t* m, size_t count, void* stream);
 
 /* Paillier::add (Eq. 5): out_i = c1_i * c2_i mod n^2.  All

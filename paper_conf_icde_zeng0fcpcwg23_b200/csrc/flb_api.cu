@@ -8,6 +8,7 @@ using namespace flb_rt;
 
 namespace flb {
 void set_last_error(const std::string& msg) { g_err = msg; }
+void set_half_units(bool on) { flb_rt::tl_half_units = on; }
 }  // namespace flb
 
 namespace {
@@ -509,10 +510,27 @@ static int pub_dev(const flb_pub* K, uint32_t** dev) { return const_cast<DevBlob
 extern "C" {
 
 // tensor-core Montgomery paths (flb_tc.cuh): on when the key has the operands; FLB_TC=0 selects
-// the CIOS kernels (read per call, so tests can compare both)
-static bool tc_enabled() {
+// the CIOS kernels, FLB_TC=2 the tensor-core kernels at every batch size (read per call, so tests
+// can compare both)
+static int tc_mode() {
   const char* e = getenv("FLB_TC");
-  return !(e && atoi(e) == 0);
+  return e ? atoi(e) : 1;
+}
+static bool tc_enabled() { return tc_mode() != 0; }
+// Public-key encryption: a tensor-core tile is 128 elements on one CTA for the whole modexp, so a
+// small batch (a few tiles on a few SMs) finishes later than the CIOS kernel spread over groups of
+// T lanes: measured crossover ≈ 12 K elements at 1024 and 2048 bits (C1's 2,000 encryptions: 8.6 ms
+// CIOS vs 16.5 ms on the tensor cores); below 96 elements per SM the CIOS kernel runs.
+static bool tc_public_batch(size_t count) {
+  const int mode = tc_mode();
+  if (mode == 0) return false;
+  if (mode == 2) return true;
+  int dev = 0, sms = 148;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+    (void)cudaGetLastError();
+    sms = 148;
+  }
+  return count >= (size_t)96 * (size_t)sms;
 }
 // FLB_TC_DAG=0: the two key-holder stages as two k_tc_exp launches instead of one k_tc_exp_dag
 static bool tc_dag_enabled() {
@@ -530,7 +548,7 @@ int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
   if (debug_checks() && (rc = check_below(m, count, K->sp, dev + K->o_n, stream, "plaintexts m >= n"))) return rc;
-  if (K->tc && tc_enabled()) {
+  if (K->tc && tc_public_batch(count)) {
     if (K->s == 128) return run_encrypt_pub_tc<128>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
     return run_encrypt_pub_tc<64>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
   }

@@ -517,6 +517,11 @@ inline int tc_tiles(flb::tc::ExpArgs& A, uint64_t* tiles, int* table) {
   return FLB_OK;
 }
 
+// Half units for a launch's incomplete last round (flb_tc.cuh): on, except while the host pipeline
+// runs concurrent chunk launches whose successors fill each other's tails (flb_host_pipeline.cu,
+// through flb::set_half_units; per calling thread)
+inline thread_local bool tl_half_units = true;
+
 inline int sm_count(int* sms) {
   int dev_id = 0;
   FLB_CK(cudaGetDevice(&dev_id));
@@ -543,6 +548,7 @@ int launch_tc_exp(flb::tc::ExpArgs& A, cudaStream_t st) {
   if (rc) return rc;
   A.scratch = (uint32_t*)s_tab.p;
   A.tab_entries = table + 1;
+  A.half_units = tl_half_units ? 1 : 0;
   flb::tc::k_tc_exp<S><<<grid, C::THREADS, C::SMEM, st>>>(A);
   FLB_LAUNCH_CHECK();
   return FLB_OK;
@@ -586,6 +592,7 @@ int launch_tc_exp_dag(flb::tc::ExpArgs& A1, flb::tc::ExpArgs& A2, cudaStream_t s
   FLB_CK(cudaMemsetAsync(s_sync.p, 0, (size_t)(1 + t1) * 4, st));
   A1.scratch = A2.scratch = (uint32_t*)s_tab.p;
   A1.tab_entries = tab1 + 1;
+  A1.half_units = A2.half_units = tl_half_units ? 1 : 0;
   A2.tab_entries = tab2 + 1;
   static_assert(flb::tc::Cfg<S1>::THREADS == flb::tc::Cfg<S2>::THREADS, "one CTA shape for both stages");
   flb::tc::k_tc_exp_dag<S1, S2><<<grid, flb::tc::Cfg<S2>::THREADS, SMEM, st>>>(A1, A2, (uint32_t*)s_sync.p, stride);

@@ -21,6 +21,7 @@
 
 namespace flb {
 void set_last_error(const std::string& msg);  // flb_api.cu: the message flb_last_error() returns
+void set_half_units(bool on);                 // flb_api.cu: half units for incomplete last rounds
 }
 
 namespace {
@@ -234,14 +235,20 @@ int flb_pack_encrypt_host_multi(const flb_pub* pub, const flb_priv* priv, const 
   }
   PCK(cudaEventRecord(C->done[0], C->st[0]));
   PCK(cudaStreamWaitEvent(C->st[1], C->done[0], 0));
-  const size_t rows = chunk_rows(total_pt), chunks = (total_pt + rows - 1) / rows;
+  // Equal chunks on two streams: chunk i+1's CTAs fill chunk i's last round, so only the final chunk
+  // ends its last round with half units (flb_tc.cuh); D2H of chunk i overlaps chunk i+1.
   const bool out_pinned = is_pinned(c_host, total_pt * ctw * 4);
+  const size_t rows = chunk_rows(total_pt), chunks = (total_pt + rows - 1) / rows;
+  struct HalfUnits {
+    ~HalfUnits() { flb::set_half_units(true); }
+  } restore;
   size_t pending_pt0 = 0, pending_n = 0;
   int pending_s = -1;
   for (size_t i = 0; i < chunks; i++) {
     const int s = (int)(i & 1);
     const size_t pt0 = i * rows, npt = std::min(rows, total_pt - pt0);
     const uint32_t* src = (const uint32_t*)C->d_mid[0].p + pt0 * ptw;
+    flb::set_half_units(i + 1 == chunks);
     int rc = priv ? flb_encrypt_crt(priv, src, nullptr, seed, ctr0 + pt0, (uint32_t*)C->d_out[s].p, npt, C->st[s])
                   : flb_encrypt(pub, src, nullptr, seed, ctr0 + pt0, (uint32_t*)C->d_out[s].p, npt, C->st[s]);
     if (rc) return lib_err(rc, "flb_encrypt");

@@ -1204,6 +1204,7 @@ struct ExpProblem {
 struct ExpArgs {
   ExpProblem pb[2];
   int nprob;
+  int half_units;          // the incomplete last round as half units (0: another launch fills the tail)
   const uint32_t* one;     // the integer 1 (at least one word)
   uint32_t* scratch;       // gridDim * kTileM * tab_entries * S words
   int tab_entries;         // max table over the problems + 1 (the per-CTA scratch stride)
@@ -1327,7 +1328,7 @@ __global__ void __launch_bounds__(Cfg<S>::THREADS, Cfg<S>::CTAS_PER_SM) k_tc_exp
   // The K tiles of an incomplete last round run as 2K half units of one product pass (≈ 0.6 of a
   // tile's time) when that still fits one round (2K <= grid): a shorter tail.
   const uint64_t rem = tiles_all % gridDim.x;
-  const uint64_t K = (C::NP == 2 && 2 * rem <= gridDim.x) ? rem : 0;
+  const uint64_t K = (A.half_units && C::NP == 2 && 2 * rem <= gridDim.x) ? rem : 0;
   const uint64_t units = tiles_all + K;
   int loaded = -1;
   uint32_t* tab = A.scratch + (size_t)blockIdx.x * kTileM * A.tab_entries * S;
@@ -1375,7 +1376,7 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
   // the last K2 stage-2 tiles (those beyond whole rounds of the grid) run as 2 K2 half units (as in
   // k_tc_exp): the queue holds T1 stage-1 tiles, then T2 - K2 stage-2 tiles, then 2 K2 half units
   const uint64_t rem2 = T2 % gridDim.x;
-  const uint64_t K2 = (Cfg<S2>::NP == 2 && 2 * rem2 <= gridDim.x) ? rem2 : 0;
+  const uint64_t K2 = (A2.half_units && Cfg<S2>::NP == 2 && 2 * rem2 <= gridDim.x) ? rem2 : 0;
   const uint64_t U2 = T2 + K2;
   int loaded = -1;  // 2 * stage + prime
   uint32_t* tab = A1.scratch + (size_t)blockIdx.x * tab_stride;

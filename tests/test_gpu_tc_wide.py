@@ -22,6 +22,8 @@ KEYS = golden_keys()
 
 
 def _env(fn, tc):
+    """FLB_TC = "0": CIOS kernels; "1": automatic (public-key encryption on the tensor cores from 96
+    elements per SM); "2": the tensor-core kernels at every batch size."""
     old = os.environ.get("FLB_TC")
     try:
         os.environ["FLB_TC"] = tc
@@ -51,7 +53,7 @@ def test_public_encrypt_tc_matches_cios_and_oracle(key, count):
         m_int[1] = n - 1
     m = to_dev(m_int, pub.pt_words)
     seed, ctr0 = 0x9B000000 + count, 5
-    tc = _env(lambda: flb.encrypt(pub, m, seed=seed, ctr0=ctr0), "1")
+    tc = _env(lambda: flb.encrypt(pub, m, seed=seed, ctr0=ctr0), "2")
     cios = _env(lambda: flb.encrypt(pub, m, seed=seed, ctr0=ctr0), "0")
     assert torch.equal(tc, cios)
     got = from_dev(tc)
@@ -72,7 +74,7 @@ def test_public_encrypt_tc_half_units(key, extra):
     per_sm = 1 if pub.ct_words >= 96 else 2  # k_tc_exp CTAs per SM (flb_tc.cuh Cfg::CTAS_PER_SM)
     count = sms * per_sm * 128 + extra
     m = to_dev(synthetic.uniform_below(n, count, 1150 + extra), pub.pt_words)
-    tc = _env(lambda: flb.encrypt(pub, m, seed=0x4A11, ctr0=2), "1")
+    tc = _env(lambda: flb.encrypt(pub, m, seed=0x4A11, ctr0=2), "2")
     cios = _env(lambda: flb.encrypt(pub, m, seed=0x4A11, ctr0=2), "0")
     bad = (tc != cios).any(dim=1).nonzero().flatten().tolist()
     assert not bad, (len(bad), bad[:5])
@@ -87,7 +89,7 @@ def test_public_encrypt_tc_caller_r_edge(key):
     ms = synthetic.uniform_below(n, len(rs), 1201)
     r = to_dev(rs, pub.pt_words)
     m = to_dev(ms, pub.pt_words)
-    tc = from_dev(_env(lambda: flb.encrypt(pub, m, r=r), "1"))
+    tc = from_dev(_env(lambda: flb.encrypt(pub, m, r=r), "2"))
     for i in range(len(rs)):
         assert tc[i] == paillier.encrypt(n, ms[i], rs[i]), i
 
