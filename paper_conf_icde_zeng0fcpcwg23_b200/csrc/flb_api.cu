@@ -329,6 +329,13 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
     case 5: {  // key-holder encryption, tensor-core kernels (k_tc_exp) only: stage 1 at H, stage 2 at sp.
       // Montgomery products on the tensor-core path; limb_products = the S^2 32x32-bit products of
       // t = a b on the IMAD pipe (the reduction's u8 MACs are 32 S^2 per product: 2 MMAs of KB^2)
+      if (V && V->tc && !V->H && sp == 32) {
+        // one stage per prime (run_encrypt_crt1_tc): 1 (entry) + table + schedule(n) + m n + final
+        const uint64_t mm = 2 * (1 + sched_mults(P->enc) + 2), sq = 2 * sched_squarings(P->enc);
+        *mont_muls = mm;
+        *limb_products = tc_imad_lp(sp, mm, sq);
+        return FLB_OK;
+      }
       if (!V || !V->tc || !V->tc_half) return fail(FLB_EUNSUPPORTED, "no tensor-core key-holder path for this key");
       const uint64_t h = V->H;
       const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
@@ -355,7 +362,9 @@ int flb_op_cost(const flb_pub* K, const flb_priv* V, int op, uint64_t* mont_muls
       uint64_t mm, lp;
       const int rc = flb_op_cost(K, V, op - 2, &mm, &lp);
       if (rc) return rc;
-      if (op == 7) {
+      if (op == 7 && !V->H) {
+        *limb_products = mm * tc_mma_macs(sp);
+      } else if (op == 7) {
         const uint64_t h = V->H;
         const uint64_t s1 = (2 + sched_mults(V->sched_q) + 1) + (2 + sched_mults(V->sched_p) + 1);
         *limb_products = s1 * tc_mma_macs(h) + (mm - s1) * tc_mma_macs(sp);
@@ -521,7 +530,7 @@ static bool tc_enabled() { return tc_mode() != 0; }
 // small batch (a few tiles on a few SMs) finishes later than the CIOS kernel spread over groups of
 // T lanes: measured crossover ≈ 12 K elements at 1024 and 2048 bits (C1's 2,000 encryptions: 8.6 ms
 // CIOS vs 16.5 ms on the tensor cores); below 96 elements per SM the CIOS kernel runs.
-static bool tc_public_batch(size_t count) {
+static bool tc_batch(size_t count) {
   const int mode = tc_mode();
   if (mode == 0) return false;
   if (mode == 2) return true;
@@ -548,7 +557,7 @@ int flb_encrypt(const flb_pub* K, const uint32_t* m, const uint32_t* r, uint64_t
   int rc = const_cast<DevBlob&>(K->dev).get(K->blob, &dev);
   if (rc) return rc;
   if (debug_checks() && (rc = check_below(m, count, K->sp, dev + K->o_n, stream, "plaintexts m >= n"))) return rc;
-  if (K->tc && tc_public_batch(count)) {
+  if (K->tc && tc_batch(count)) {
     if (K->s == 128) return run_encrypt_pub_tc<128>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
     return run_encrypt_pub_tc<64>(K, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
   }
@@ -594,6 +603,9 @@ int flb_encrypt_crt(const flb_priv* V, const uint32_t* m, const uint32_t* r, uin
       return rc;
   }
   if (V->H) return encrypt_crt_v2(V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
+  // one stage per prime (1024-bit keys): (1 + m n) r^n mod P^2 on the tensor cores for large batches
+  if (V->tc && V->pub->sp == 32 && tc_batch(count))
+    return run_encrypt_crt1_tc<32>(V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
   FLB_DISPATCH_DEC(V->pub->frame, run_encrypt_crt, V, dev, m, r, seed, ctr0, c, count, (cudaStream_t)stream);
 }
 

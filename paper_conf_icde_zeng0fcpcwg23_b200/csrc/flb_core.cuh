@@ -716,6 +716,50 @@ inline int philox_fill(uint32_t sp, uint32_t nbits, uint64_t seed, uint64_t ctr0
 // public-key encryption on the tensor cores (Eq. 3): c = (1 + m n) r^n mod n^2 in the
 // S = ct_words frame, every Montgomery product of the modexp with its reduction as u8 MMAs against
 // the Toeplitz operands of n^2 (one problem, k_tc_exp<S>)
+// key-holder encryption in one stage on the tensor cores (keys without a half frame, 1024 bits):
+// c_P = (1 + m n) r^n mod P^2 for both primes in one k_tc_exp launch (x = r < n < R enters the
+// Montgomery domain by one product with R^2), then k_crt_combine; r drawn as k_encrypt_crt does
+template <int S>
+int run_encrypt_crt1_tc(const flb_priv* V, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
+                        uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
+  const flb_pub* K = V->pub;
+  Scratch s_r, s_out;
+  int rc;
+  if (!r) {
+    rc = philox_fill(K->sp, K->nbits, seed, ctr0, count, s_r, st);
+    if (rc) return rc;
+    r = (const uint32_t*)s_r.p;
+  }
+  rc = s_out.alloc((size_t)2 * count * S * 4, st);
+  if (rc) return rc;
+  uint32_t* cpq = (uint32_t*)s_out.p;
+  flb::tc::ExpArgs A{};
+  A.nprob = 2;
+  A.one = dev + V->o_one;
+  for (int i = 0; i < 2; i++) {
+    const auto& R = V->pr[i];
+    auto& P = A.pb[i];
+    P.N = dev + R.o_P2;
+    P.R2 = dev + R.o_R2;
+    P.R3 = dev + R.o_R3;
+    P.E1 = dev + R.o_tcE1;
+    P.E2 = dev + R.o_tcE2;
+    P.sched = dev + V->o_enc_sched;  // exponent n
+    P.sched_len = (int)K->enc.ops.size();
+    P.table = K->enc.table;
+    P.x = r;
+    P.x_stride = P.x_words = K->sp;
+    P.m = m;
+    P.m_stride = P.m_words = K->sp;
+    P.nR = dev + R.o_nR;
+    P.out = cpq + (size_t)i * count * S;
+    P.count = count;
+  }
+  rc = launch_tc_exp<S>(A, st);
+  if (rc) return rc;
+  return tc_combine<S>(V, dev, cpq, c, count, st);
+}
+
 template <int S>
 int run_encrypt_pub_tc(const flb_pub* K, const uint32_t* dev, const uint32_t* m, const uint32_t* r, uint64_t seed,
                        uint64_t ctr0, uint32_t* c, size_t count, cudaStream_t st) {
@@ -1022,6 +1066,9 @@ int run_reduce(const flb_pub* K, const uint32_t* dev, const uint32_t* c, size_t 
   EXT template int flb_rt::run_encrypt_crt2<X, T>(const flb_priv*, const uint32_t*, const uint32_t*,             \
                                                   const uint32_t*, uint32_t*, size_t, cudaStream_t);
 #define FLB_TC_DECLS(EXT, S)                                                                                      \
+  EXT template int flb_rt::run_encrypt_crt1_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*,             \
+                                                  const uint32_t*, uint64_t, uint64_t, uint32_t*, size_t,        \
+                                                  cudaStream_t);                                                  \
   EXT template int flb_rt::run_encrypt_crt_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*,              \
                                                  const uint32_t*, uint32_t*, size_t, cudaStream_t);              \
   EXT template int flb_rt::run_crt_pre_tc<S>(const flb_priv*, const uint32_t*, const uint32_t*, uint64_t,        \

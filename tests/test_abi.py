@@ -228,8 +228,13 @@ def test_op_cost_tensor_core_paths():
     assert any(lp_e == (s1 - a - b) * h * h + (a + b) * sq32
                + (s2 - a - b) * sp * sp + (a + b) * sq64 for a in esp for b in esq)
     assert flb.op_cost(priv, "encrypt_crt_tc_macs") == (mm_e, s1 * macs(h) + s2 * macs(sp))
-    # 1024-bit keys have no two-stage (half-frame) encryption path
+    # 1024-bit keys have no two-stage (half-frame) path: one stage per prime, (1 + m n) r^n mod P^2 with
+    # the exponent n in the 32-word frame (entry, table + schedule of n, m n, final product)
     p1, q1 = KEYS["1024"]
     _, priv1 = flb.key_from_primes(p1, q1)
-    with pytest.raises(flb.FlbError):
-        flb.op_cost(priv1, "encrypt_crt_tc")
+    mm1, lp1 = flb.op_cost(priv1, "encrypt_crt_tc")
+    (mn, sqn) = best(p1 * q1)
+    assert mm1 == 2 * (1 + mn + 2)
+    sq32 = 2 * (X * (X + 1) // 2 + X * X // 2)
+    assert any(lp1 == (mm1 - 2 * a) * 32 * 32 + 2 * a * sq32 for a in sqn)
+    assert flb.op_cost(priv1, "encrypt_crt_tc_macs") == (mm1, mm1 * macs(32))

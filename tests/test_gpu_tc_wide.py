@@ -147,3 +147,27 @@ def test_tc_product_phase_128():
     for i in range(count):
         assert t[i] == a_int[i] * b_int[i], i
         assert t2[i] == a_int[i] * a_int[i], i
+
+
+@pytest.mark.parametrize("count", [1, 129, 300, 20000])
+def test_keyholder_encrypt_1024_one_stage_tc(count):
+    """1024-bit key-holder encryption (no half frame): (1 + m n) r^n mod P^2 for both primes on the S = 32
+    tensor-core kernel (exponent n), then the CRT recombination; same bits as the CIOS k_encrypt_crt and
+    as the oracle's Eq. 3 (20,000 elements: the automatic dispatch takes the tensor cores too)."""
+    p, q = KEYS["1024"]
+    pub, priv = flb.key_from_primes(p, q)
+    n = p * q
+    m_int = synthetic.uniform_below(n, count, 1600 + count)
+    m_int[0] = 0
+    if count > 1:
+        m_int[-1] = n - 1
+    m = to_dev(m_int, pub.pt_words)
+    tc = _env(lambda: flb.encrypt_crt(priv, m, seed=31, ctr0=4), "2")
+    cios = _env(lambda: flb.encrypt_crt(priv, m, seed=31, ctr0=4), "0")
+    assert torch.equal(tc, cios)
+    if count >= 20000:
+        auto = _env(lambda: flb.encrypt_crt(priv, m, seed=31, ctr0=4), "1")
+        assert torch.equal(auto, cios)
+    got = from_dev(tc)
+    for i in sorted({0, count // 2, count - 1}):
+        assert got[i] == paillier.encrypt(n, m_int[i], philox.draw_r(n, 31, 4 + i, pub.pt_words)), i

@@ -16,7 +16,7 @@ for bits,count in ((2048,133160),(1024,133160),(3072,16384),(4096,16384)):
     for tc in ("1","0"):
         os.environ["FLB_TC"]=tc
         out["%d_pub_enc_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.encrypt(pub,m,seed=3)))
-        if bits>=3072:
+        if bits>=3072 or bits==1024:
             c=flb.encrypt_crt(priv,m,seed=3)
             out["%d_dec_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.decrypt(priv,c)))
             out["%d_kh_enc_tc%s_per_s"%(bits,tc)]=round(count/timed(lambda: flb.encrypt_crt(priv,m,seed=3)))
