@@ -235,7 +235,10 @@ def run_reference(args):
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32-limb bigint (+f64 codec)",
         "data": "synthetic",
         "config": {"workload": "C2 Homo-LR aggregation, 2048-bit key, 8 clients x 1,048,576 values",
-                   "note": "CPU oracle: each step times a bounded sample and extrapolates to the C2 step"},
+                   "note": "CPU oracle: each step times a bounded sample (about %.0f s of CPU work) and "
+                           "extrapolates to the C2 step; ms_per_step is that extrapolated step time, not the "
+                           "wall clock of this run" % per},
+        "ms_per_step_extrapolated": True,
         "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": vals[-1][2]},
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
