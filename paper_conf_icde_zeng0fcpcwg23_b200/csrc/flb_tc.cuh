@@ -897,7 +897,9 @@ __device__ __forceinline__ void tc_product(const Src& sa, const Src& sb, bool sq
 
 // Montgomery product over the tile: for every element, a b R^-1 mod N (canonical) into its work
 // row.  sq: b = a.  `phase` tracks the mbarrier parity (two completions per call).  CTA-collective.
-template <int S, int SQ = FLB_TC_TRISQ>
+// LDP: the normalisation double-buffers its TMEM loads (chunk c + 1 in flight while chunk c is
+// normalised) — measured faster in k_tc_exp_dag (245.4 -> 242.1 ms), slower in k_tc_exp.
+template <int S, int SQ = FLB_TC_TRISQ, bool LDP = false>
 __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, const Smem& sm,
                                         const uint32_t* __restrict__ Nmod, uint32_t& phase) {
   using C = Cfg<S>;
@@ -964,12 +966,27 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
   // ---- N1: q = D1 mod R
   if (nw) {
     NormState ns;
-#pragma unroll
-    for (int c0 = 0; c0 < QC; c0 += 32) {
-      uint32_t cv[32];
-      tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
+    if constexpr (LDP) {
+      // the TMEM load of chunk c + 1 is in flight while chunk c is normalised (two 32-column buffers)
+      uint32_t ca[32], cb[32];
+      tmem_ld32(lane_base + (uint32_t)(g * QC), ca);
       tmem_wait();
-      norm8_chain<false>(cv, nullptr, v + c0 / 4, ns, c0 == 0);
+#pragma unroll
+      for (int c0 = 0; c0 < QC; c0 += 32) {
+        uint32_t(&cur)[32] = ((c0 / 32) & 1) ? cb : ca;
+        uint32_t(&nxt)[32] = ((c0 / 32) & 1) ? ca : cb;
+        if (c0 + 32 < QC) tmem_ld32(lane_base + (uint32_t)(g * QC + c0 + 32), nxt);
+        norm8_chain<false>(cur, nullptr, v + c0 / 4, ns, c0 == 0);
+        if (c0 + 32 < QC) tmem_wait();
+      }
+    } else {
+#pragma unroll
+      for (int c0 = 0; c0 < QC; c0 += 32) {
+        uint32_t cv[32];
+        tmem_ld32(lane_base + (uint32_t)(g * QC + c0), cv);
+        tmem_wait();
+        norm8_chain<false>(cv, nullptr, v + c0 / 4, ns, c0 == 0);
+      }
     }
     publish(ns.carry_out_end());
   }
@@ -1033,28 +1050,66 @@ __device__ __forceinline__ void tc_mont(const Src& sa, const Src& sb, bool sq, c
         top[j] = acc;
       }
     }
+    if constexpr (LDP) {
+      // as N1: chunk c + 1's TMEM loads overlap chunk c's normalisation
+      auto load_chunk = [&](int c0, uint32_t(&cv)[32], uint32_t(&t8)[8]) {
+        const uint32_t col = 8u + (uint32_t)(g * QC + c0);
+        if (c0 + 32 < QC) {
+          tmem_ld32(lane_base + col, cv);
+        } else {  // D2 columns col + 24 .. col + 31 exist for all but the last group (its top columns)
+          tmem_ld16(lane_base + col, cv);
+          tmem_ld8(lane_base + col + 16u, cv + 16);
+          tmem_ld8(lane_base + (g < NG - 1 ? col + 24u : 0u), t8);  // uniform per warp; unused for the last
+        }
+      };
+      auto fix_last = [&](int c0, uint32_t(&cv)[32], const uint32_t(&t8)[8]) {
+        if (c0 + 32 >= QC) {
 #pragma unroll
-    for (int c0 = 0; c0 < QC; c0 += 32) {
-      uint32_t cv[32];
-      const uint32_t col = 8u + (uint32_t)(g * QC + c0);
-      if (c0 + 32 < QC) {
-        tmem_ld32(lane_base + col, cv);
-      } else {
-        // last chunk of the group: D2 columns col .. col+23 always exist; col+24 .. col+31 exist
-        // for all but the last group (whose are the top columns)
-        tmem_ld16(lane_base + col, cv);
-        tmem_ld8(lane_base + col + 16u, cv + 16);
-        uint32_t t8[8];
-        tmem_ld8(lane_base + (g < NG - 1 ? col + 24u : 0u), t8);  // uniform per warp; unused for the last
-        tmem_wait();
-#pragma unroll
-        for (int j = 0; j < 8; j++) cv[24 + j] = g < NG - 1 ? t8[j] : top[j];
-      }
+          for (int j = 0; j < 8; j++) cv[24 + j] = g < NG - 1 ? t8[j] : top[j];
+        }
+      };
+      uint32_t ca[32], cb[32], t8[8];
+      load_chunk(0, ca, t8);
       tmem_wait();
-      const uint4 h0 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[0];  // 8 words, one 32-block
-      const uint4 h1 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[1];
-      const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
-      norm8_chain<true>(cv, th, v + c0 / 4, ns, c0 == 0);
+      fix_last(0, ca, t8);
+#pragma unroll
+      for (int c0 = 0; c0 < QC; c0 += 32) {
+        uint32_t(&cur)[32] = ((c0 / 32) & 1) ? cb : ca;
+        uint32_t(&nxt)[32] = ((c0 / 32) & 1) ? ca : cb;
+        if (c0 + 32 < QC) load_chunk(c0 + 32, nxt, t8);
+        const uint4 h0 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[0];  // 8 words, one 32-block
+        const uint4 h1 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[1];
+        const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
+        norm8_chain<true>(cur, th, v + c0 / 4, ns, c0 == 0);
+        if (c0 + 32 < QC) {
+          tmem_wait();
+          fix_last(c0 + 32, nxt, t8);
+        }
+      }
+    } else {
+#pragma unroll
+      for (int c0 = 0; c0 < QC; c0 += 32) {
+        uint32_t cv[32];
+        const uint32_t col = 8u + (uint32_t)(g * QC + c0);
+        if (c0 + 32 < QC) {
+          tmem_ld32(lane_base + col, cv);
+        } else {
+          // last chunk of the group: D2 columns col .. col+23 always exist; col+24 .. col+31 exist
+          // for all but the last group (whose are the top columns)
+          tmem_ld16(lane_base + col, cv);
+          tmem_ld8(lane_base + col + 16u, cv + 16);
+          uint32_t t8[8];
+          tmem_ld8(lane_base + (g < NG - 1 ? col + 24u : 0u), t8);  // uniform per warp; unused for the last
+          tmem_wait();
+#pragma unroll
+          for (int j = 0; j < 8; j++) cv[24 + j] = g < NG - 1 ? t8[j] : top[j];
+        }
+        tmem_wait();
+        const uint4 h0 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[0];  // 8 words, one 32-block
+        const uint4 h1 = reinterpret_cast<const uint4*>(row + wpad<S>(g * QW + c0 / 4))[1];
+        const uint32_t th[8] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
+        norm8_chain<true>(cv, th, v + c0 / 4, ns, c0 == 0);
+      }
     }
     publish(ns.carry_out_end());
   }
@@ -1227,7 +1282,7 @@ __device__ __forceinline__ void tc_load_operands(uint8_t* smem, const ExpProblem
 // is the CTA's window-table scratch ([entry][kTileM][S] words).  The Toeplitz operands of P are in
 // shared memory (tc_load_operands).  hf >= 0: half unit hf of the tile (its elements 64 hf .. 64 hf + 63
 // on the rows of product pass 0, sm.np = 1).
-template <int S, int SQ = FLB_TC_TRISQ>
+template <int S, int SQ = FLB_TC_TRISQ, bool LDP = false>
 __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, const uint32_t* one, uint32_t* tab,
                                             const Smem& sm, uint32_t& phase, uint32_t x_ld = kLdNC, int hf = -1) {
   const Src row = src_row();
@@ -1241,22 +1296,22 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
   const uint32_t nvalid = e0 >= P.count ? 0u : (uint32_t)((P.count - e0) < cap ? (P.count - e0) : cap);
   const uint32_t* xb = P.x + e0 * P.x_stride;
   if (P.x_words <= (uint32_t)S) {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, P.x_words, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm,
+    tc_mont<S, SQ, LDP>(src_arr(xb, P.x_stride, P.x_words, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm,
                    P.N, phase);
   } else {
-    tc_mont<S, SQ>(src_arr(xb, P.x_stride, S, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
+    tc_mont<S, SQ, LDP>(src_arr(xb, P.x_stride, S, nvalid, x_ld, half), src_arr(P.R2, 0, S, kTileM), false, sm, P.N, phase);
     tc_row_store<S>(sm, slot_ptr(0), S, kTileM);            // lo R
-    tc_mont<S, SQ>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid, x_ld, half), src_arr(P.R3, 0, S, kTileM), false,
+    tc_mont<S, SQ, LDP>(src_arr(xb + S, P.x_stride, P.x_words - S, nvalid, x_ld, half), src_arr(P.R3, 0, S, kTileM), false,
                    sm, P.N, phase);                         // hi R^2
     tc_row_add<S>(sm, slot(0), P.N);
   }
   tc_row_store<S>(sm, slot_ptr(0), S, kTileM);              // x R mod N
   if (TB > 1) {
-    tc_mont<S, SQ>(row, row, true, sm, P.N, phase);             // x^2
+    tc_mont<S, SQ, LDP>(row, row, true, sm, P.N, phase);             // x^2
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);
 #pragma unroll 1
     for (int t = 1; t < TB; t++) {
-      tc_mont<S, SQ>(slot(t - 1), slot(TB), false, sm, P.N, phase);
+      tc_mont<S, SQ, LDP>(slot(t - 1), slot(TB), false, sm, P.N, phase);
       tc_row_store<S>(sm, slot_ptr(t), S, kTileM);
     }
   }
@@ -1268,22 +1323,22 @@ __device__ __forceinline__ void tc_exp_tile(const ExpProblem& P, uint64_t tile, 
     const int sq = (int)(op & 0xffffu), idx = (int)(op >> 16) - 1;
 #pragma unroll 1
     for (int t = 0; t < sq; t++) {
-      tc_mont<S, SQ>(cur, cur, true, sm, P.N, phase);
+      tc_mont<S, SQ, LDP>(cur, cur, true, sm, P.N, phase);
       cur = row;
     }
     if (idx >= 0) {
-      tc_mont<S, SQ>(cur, slot(idx), false, sm, P.N, phase);
+      tc_mont<S, SQ, LDP>(cur, slot(idx), false, sm, P.N, phase);
       cur = row;
     }
   }
   if (P.m) {
     tc_row_store<S>(sm, slot_ptr(TB), S, kTileM);           // x^E R
-    tc_mont<S, SQ>(src_arr(P.m + e0 * P.m_stride, P.m_stride, P.m_words, nvalid, kLdNC, half),
+    tc_mont<S, SQ, LDP>(src_arr(P.m + e0 * P.m_stride, P.m_stride, P.m_words, nvalid, kLdNC, half),
                    src_arr(P.nR, 0, S, kTileM), false, sm, P.N, phase);  // m n
     tc_row_add_one<S>(sm, P.N);                             // 1 + m n mod N
-    tc_mont<S, SQ>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
+    tc_mont<S, SQ, LDP>(slot(TB), row, false, sm, P.N, phase);       // (1 + m n) x^E
   } else {
-    tc_mont<S, SQ>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
+    tc_mont<S, SQ, LDP>(row, src_arr(one, 0, 1, kTileM), false, sm, P.N, phase);  // leave the Montgomery domain
   }
   tc_row_store<S>(sm, P.out + e0 * S, S, nvalid, half);
 }
@@ -1412,9 +1467,9 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
       }
       __syncthreads();
       // y: written by another CTA of this launch
-      tc_exp_tile<S2, FLB_TC_TRISQ_S2>(P, tile, A2.one, tab, whole ? sm2 : sm2h, phase, kLdGPU, hf);
+      tc_exp_tile<S2, FLB_TC_TRISQ_S2, true>(P, tile, A2.one, tab, whole ? sm2 : sm2h, phase, kLdGPU, hf);
     } else {
-      tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm1, phase);
+      tc_exp_tile<S1, FLB_TC_TRISQ_S1, true>(P, tile, A1.one, tab, sm1, phase);
     }
     __syncthreads();  // the tile's output rows are stored; the work rows are rewritten next
     if (threadIdx.x == 0) {
