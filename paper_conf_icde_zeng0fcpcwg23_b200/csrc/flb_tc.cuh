@@ -414,7 +414,7 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 #define FLB_TC_TRISQ 1  // diagonal blocks a_k^2: 1 = one lane-local triangular square, 2 = the half-split form
 #endif
 #ifndef FLB_TC_TRISQ_S1
-#define FLB_TC_TRISQ_S1 2  // stage-1 tiles (S = 32) of k_tc_exp_dag: the half-split form
+#define FLB_TC_TRISQ_S1 1  // stage-1 tiles (S = 32) of k_tc_exp_dag: one triangle (measured with the double-buffered loads)
 #endif
 #ifndef FLB_TC_TRISQ_S2
 #define FLB_TC_TRISQ_S2 1  // stage-2 tiles (S = 64) of k_tc_exp_dag
