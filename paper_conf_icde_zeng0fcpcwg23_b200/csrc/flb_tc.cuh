@@ -420,7 +420,7 @@ __device__ __forceinline__ void blk_prod(uint32_t (&out)[X + R], const uint32_t 
 #define FLB_TC_TRISQ_S2 1  // stage-2 tiles (S = 64) of k_tc_exp_dag
 #endif
 #ifndef FLB_TC_TRISQ_EXP
-#define FLB_TC_TRISQ_EXP 2  // k_tc_exp (decryption; two-launch key-holder stages): the half-split form
+#define FLB_TC_TRISQ_EXP 1  // k_tc_exp (decryption, public, two-launch key-holder stages): one triangle
 #endif
 
 // v = a^2 (2X words) for this lane's own block, X (X - 1) / 2 + X limb products instead of X^2
