@@ -1469,7 +1469,7 @@ __global__ void __launch_bounds__(Cfg<S2>::THREADS, 2) k_tc_exp_dag(const ExpArg
       // y: written by another CTA of this launch
       tc_exp_tile<S2, FLB_TC_TRISQ_S2, true>(P, tile, A2.one, tab, whole ? sm2 : sm2h, phase, kLdGPU, hf);
     } else {
-      tc_exp_tile<S1, FLB_TC_TRISQ_S1, true>(P, tile, A1.one, tab, sm1, phase);
+      tc_exp_tile<S1, FLB_TC_TRISQ_S1>(P, tile, A1.one, tab, sm1, phase);  // (single-buffered loads: measured)
     }
     __syncthreads();  // the tile's output rows are stored; the work rows are rewritten next
     if (threadIdx.x == 0) {
